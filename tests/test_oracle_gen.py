@@ -1,0 +1,159 @@
+"""Pins for the oracle's generator (O-GEN) and shard map (O-SHARD) -- SURVEY §8(c), docs/GENERATOR.md.
+
+What pins them (other than the oracle itself):
+  * splitmix64 published reference vectors (Vigna's splitmix64.c, seed 1234567);
+  * exact rational arithmetic for pm1 (Python Fractions);
+  * brute-force invariants of the row distribution, shard map (numpy.searchsorted = lower_bound), and of the
+    paper's storage structure (5 contiguous astro columns at 5*star; 3 attitude blocks of 4 with a
+    fixed stride; 6 instrumental columns);
+  * planted b equals the dense product A @ x_true;
+  * golden checksums (tests/golden/gen_checksums.json, written by tests/golden/make_golden.py from the oracle).
+"""
+import json
+import os
+from fractions import Fraction
+
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+from tests.golden.make_golden import golden_cases, system_checksums
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden", "gen_checksums.json")
+
+
+def test_splitmix64_reference_vectors():
+    # splitmix64 generator output k = mix(seed + k*gamma) (our mix adds gamma first, so output k is
+    # mix(seed + k*gamma)).  Reference: first five outputs for seed 1234567 from the published splitmix64.c.
+    ref = [6457827717110365317, 3203168211198807973, 9817491932198370423, 4593380528125082431,
+           16408922859458223821]
+    G = 0x9E3779B97F4A7C15
+    got = [oracle.lib().orc_mix((1234567 + k * G) % 2**64) for k in range(5)]
+    assert got == ref
+
+
+def test_hash_composition():
+    L = oracle.lib()
+    for seed, tag, i, j in [(1, 4, 0, 0), (20241117, 2, 123456789, 0), (7, 8, 5, 99)]:
+        h = L.orc_mix(L.orc_mix(L.orc_mix(seed ^ (tag << 56)) ^ i) ^ j)
+        assert oracle.hash64(seed, tag, i, j) == h
+
+
+def test_pm1_exact_and_range():
+    for h in [0, 1, 2**10 - 1, 2**10, 2**63, 2**64 - 1, 0xDEADBEEFCAFEBABE]:
+        want = Fraction((h >> 10) - 2**53, 2**53)
+        got = oracle.pm1(h)
+        assert Fraction(got) == want
+        assert -1.0 <= got < 1.0
+    assert oracle.pm1(0) == -1.0
+    assert oracle.pm1(2**64 - 1) == 1.0 - 2.0**-53
+
+
+@pytest.mark.parametrize("n_stars,n_obs,pct", [(1000, 20000, 0), (1001, 20007, 0), (50, 5000, 50), (51, 5003, 50),
+                                               (10, 15, 50), (5, 3, 50), (7, 700, 100)])
+def test_star_counts(n_stars, n_obs, pct):
+    w = W.Workload("t", n_stars=n_stars, n_obs=n_obs, n_att=12, n_instr=6, jitter_pct=pct, seed=11)
+    c = oracle.star_counts(w)
+    assert c.sum() == n_obs
+    q, rem = divmod(n_obs, n_stars)
+    base = np.array([q + (s < rem) for s in range(n_stars)])
+    J = (q * pct) // 100
+    if q == 0:
+        J = 0
+    elif q - J < 1:
+        J = q - 1
+    if J == 0:
+        assert (c == base).all()
+        return
+    npairs = n_stars // 2
+    d = c[: 2 * npairs: 2] - base[: 2 * npairs: 2]
+    assert (c[1: 2 * npairs: 2] - base[1: 2 * npairs: 2] == -d).all()
+    assert np.abs(d).max() <= J
+    if n_stars % 2:
+        assert c[-1] == base[-1]
+    if q >= 1:
+        assert (c >= 1).all()
+    # the jitter is actually exercised
+    assert len(np.unique(d)) > 1 or npairs < 3
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
+def test_shard_lower_bound_cover_disjoint(P):
+    w = W.C2.replace(n_stars=5000, n_obs=500_000)
+    rp = oracle.row_ptr(oracle.star_counts(w))
+    sb = oracle.shard(rp, w.n_obs, P)
+    assert sb[0] == 0 and sb[P] == w.n_stars
+    assert (np.diff(sb) >= 0).all()
+    for r in range(1, P):
+        target = (r * w.n_obs) // P
+        assert sb[r] == np.searchsorted(rp, target, side="left")
+    rows = [rp[sb[r + 1]] - rp[sb[r]] for r in range(P)]
+    assert sum(rows) == w.n_obs
+    # balanced by rows to within one star
+    assert max(rows) - min(rows) <= 2 * int(np.diff(rp).max())
+
+
+def test_golden_checksums():
+    with open(GOLDEN) as f:
+        gold = json.load(f)
+    for name, w in golden_cases().items():
+        S = oracle.System(w)
+        assert system_checksums(S) == gold[name], name
+
+
+@pytest.mark.parametrize("w", [W.micro(), W.micro(n_glob=0, seed=5), W.micro(n_stars=13, obs=25, n_att=36,
+                                                                              n_instr=18, n_ext=5, seed=8)])
+def test_structure_invariants(w):
+    S = oracle.System(w)
+    n_axis, g = w.n_att // 3, w.n_instr // 6
+    stars = np.repeat(np.arange(w.n_stars), oracle.star_counts(w))
+    assert (S.mA == 5 * stars).all()                                   # block diagonal astro
+    k0 = S.mT - S.A0
+    assert k0.min() >= 0 and k0.max() <= n_axis - 4                     # 3 blocks of 4, stride n_axis
+    for j in range(6):                                                   # one instr column per group
+        rel = S.iC[:, j] - S.I0
+        assert rel.min() >= j * g and rel.max() < (j + 1) * g
+    assert (S.vals >= -1).all() and (S.vals < 1).all()
+    if w.n_glob == 0:
+        assert (S.vals[:, 23] == 0).all()
+    assert (S.b >= -1).all() and (S.b < 1).all()
+
+
+@pytest.mark.parametrize("P", [2, 3, 4])
+def test_sharded_generation_is_slice_of_full(P):
+    w = W.micro(n_stars=11, obs=20, n_ext=3, seed=21)
+    full = oracle.System(w)
+    for r in range(P):
+        S = oracle.System(w, rank=r, nranks=P)
+        sl = slice(S.row_begin, S.row_end)
+        for name in ("vals", "mA", "mT", "iC", "b"):
+            assert np.array_equal(getattr(S, name), getattr(full, name)[sl]), name
+
+
+def test_planted_b_is_A_xtrue():
+    w = W.micro(seed=13, b_mode=1, noise=0.0)
+    S = oracle.System(w)
+    A = S.dense()[: S.n_rows]
+    xt = oracle.x_true(w)
+    ref = A @ xt
+    scale = np.abs(A) @ np.abs(xt)
+    assert (np.abs(S.b - ref) <= 1e-14 * scale).all()
+    w2 = w.replace(noise=0.5)
+    S2 = oracle.System(w2)
+    e = S2.b - S.b
+    assert np.abs(e).max() <= 0.5 + 1e-15 and np.abs(e).max() > 0.1
+
+
+def test_constraints_structure():
+    w = W.C1C
+    ptr, col, val = oracle.constraints(w)
+    assert len(ptr) == 13 and ptr[-1] == len(col) == 6 * 5 * 1000 + w.n_instr
+    for k in range(6):
+        c = col[ptr[k]:ptr[k + 1]]
+        assert (c == np.arange(5000)).all()
+    g = w.n_instr // 6
+    for j in range(6):
+        c = col[ptr[6 + j]:ptr[7 + j]]
+        assert (c == 5 * w.n_stars + w.n_att + j * g + np.arange(g)).all()
+        assert (val[ptr[6 + j]:ptr[7 + j]] == 1.0).all()
