@@ -1,0 +1,332 @@
+#!/usr/bin/env python
+"""Benchmark: seconds per LSQR iteration and HBM-roofline fraction (FP64) of the AVU-GSR hot path on B200.
+
+    python bench.py [--gpus N --steps K --warmup W --config C2]          # our CUDA path (one JSON line)
+    python bench.py --impl reference ...                                  # the CPU oracle (reference arm)
+    torchrun --nproc-per-node N bench.py --gpus N ...                     # multi-GPU, weak scaling
+
+A "step" is one LSQR iteration (aprod1 + beta + aprod2 + shared-slice update + scalar recurrence + column update,
+SURVEY §8(a) a3-a9) over the whole synthetic system; in fixed-count mode as in the paper.  Weak
+scaling: every GPU holds one copy of the configuration's shape (n_stars, n_obs multiplied by N).  Inputs (A: 1 GB
+at C2) are larger than L2 (126 MB), so no L2 flush is needed between iterations.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import workloads as W  # noqa: E402
+
+METRIC = "s per LSQR iteration & % of HBM roofline (FP64) at 1/2/4/8 B200"
+UNIT = "s/iteration"
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+# ------------------------------------------------------------------------------------------------ clocks
+class ClockSampler:
+    """Samples SM clock and throttle reasons during the timed region (pynvml; nvidia-smi fallback)."""
+
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+               0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, device=0, period=0.05):
+        self.device, self.period = device, period
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self._stop = threading.Event()
+        self._t = None
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            self.nv = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self.REASONS.items():
+                    if r & bit and name != "gpu_idle":
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+# ------------------------------------------------------------------------------------------------ bytes
+def algorithmic_bytes(w, n_rows, n_stars, n_sh, n_cols):
+    """Algorithmic HBM bytes per launch.
+    aprod1: A values 192 B + index record 16 B + u read 8 B + u write 8 B per row; v_astro 40 B per star; v_shared
+    gathered once (8 B per shared column).  aprod2: 192 + 16 + 8 (u) per row; v_astro read+write 80 B per star;
+    z_shared written once.  Iteration (two-pass): both products + column update (v, w, x, var read, v, w, x, var
+    written: 7 x 8 B per column counted as in SURVEY: 56 B) -- 440 B/row + 56 B/column."""
+    ap1 = 224 * n_rows + 40 * n_stars + 8 * n_sh
+    ap2 = 216 * n_rows + 80 * n_stars + 8 * n_sh
+    it = 440 * n_rows + 56 * n_cols
+    return ap1, ap2, it
+
+
+def load_traffic(kernel):
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return d.get(kernel)
+    return None
+
+
+# ------------------------------------------------------------------------------------------------ cpu baseline
+def cpu_baseline(w, iters=3):
+    """The oracle (serial C, as it stands) on a bounded sample: the full system, `iters` LSQR iterations."""
+    import oracle
+    t0 = time.perf_counter()
+    S = oracle.System(w)
+    S.apply_precond()
+    t_setup = time.perf_counter() - t0
+    stamps = []
+    oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), atol=0, btol=0, conlim=0, itn_limit=iters + 1, fixed_count=True,
+                want_se=False, trace=lambda st: stamps.append(time.perf_counter()), trace_vectors=False)
+    per = [b - a for a, b in zip(stamps[:-1], stamps[1:])]
+    v = float(np.median(per))
+    return {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"full {w.name} system ({w.n_obs} rows), {len(per)} timed LSQR iterations of the serial C "
+                      f"oracle after 1 untimed (setup {t_setup:.1f} s excluded)",
+            "cpu_model": _cpu_model(), "host_cores": os.cpu_count()}
+
+
+def _cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return None
+
+
+def config_block(w, n, args, extra=None):
+    c = {"workload": w.name, "n_stars_per_gpu": w.n_stars, "n_obs_per_gpu": w.n_obs, "n_att": w.n_att,
+         "n_instr": w.n_instr, "n_glob": w.n_glob, "constraint_rows": w.n_constr, "obs_jitter_pct": w.jitter_pct,
+         "A_bytes_per_gpu": w.a_bytes, "preconditioned": True, "mode": "fixed-count (paper timing mode)",
+         "seed": w.seed, "parallelism": f"dp{n} (rows sharded by star)",
+         "l2": "no flush: A per GPU (%.2f GB) >> L2 (126 MB)" % (w.a_bytes / 1e9)}
+    if extra:
+        c.update(extra)
+    return c
+
+
+# ------------------------------------------------------------------------------------------------ reference arm
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    base = W.CONFIGS[args.config]
+    w = base
+    import oracle
+    t0 = time.perf_counter()
+    S = oracle.System(w)
+    S.apply_precond()
+    setup = time.perf_counter() - t0
+    stamps = [time.perf_counter()]
+    oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), atol=0, btol=0, conlim=0, itn_limit=args.warmup + args.steps,
+                fixed_count=True, want_se=False, trace=lambda st: stamps.append(time.perf_counter()),
+                trace_vectors=False)
+    per = [b - a for a, b in zip(stamps[:-1], stamps[1:])][args.warmup:]
+    v = float(np.mean(per))
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": len(per), "warmup": args.warmup, "ms_per_step": v * 1e3, "higher_is_better": False,
+            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": config_block(w, 1, args, {"note": "CPU oracle (serial C, -O2 -ffp-contract=off) on the host; "
+                                                        "rank 0 only"}),
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
+                             "sample": f"full {w.name} system, {len(per)} LSQR iterations after {args.warmup} "
+                                       f"warm-up (setup {setup:.1f} s excluded)", "cpu_model": _cpu_model()},
+            "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------------------------------------ our arm
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_sc_malenzacsbvba24_b200 as avu
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    n = world
+    torch.cuda.set_device(local)
+    multi = world > 1
+    if multi:
+        dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", local))
+    base = W.CONFIGS[args.config]
+    w = base.per_gpu(n) if n > 1 else base
+    w = w.replace(name=base.name)
+    kw = {}
+    if multi:
+        obj = [avu.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        kw = dict(comm="nccl", nccl_id=obj[0])
+    K, Wm = args.steps, args.warmup
+
+    def barrier():
+        if multi:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def max_over_ranks(v):
+        if not multi:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    # ---------------- e2e through the public API with HOST buffers (set_system -> precondition -> solve -> x, se)
+    e2e = None
+    if args.e2e:
+        s0 = avu.Solver.synthetic(base.per_gpu(n).replace(name=base.name) if n > 1 else base, rank=rank,
+                                  nranks=world, **kw)
+        g = s0.get_system()
+        nloc_cols = s0.n_local_cols
+        s0.close()
+        torch.cuda.synchronize()
+        pin = {k: torch.from_numpy(np.ascontiguousarray(v)).pin_memory() for k, v in g.items()}
+        del g
+        xo = torch.empty(nloc_cols, dtype=torch.float64).pin_memory()
+        so = torch.empty(nloc_cols, dtype=torch.float64).pin_memory()
+        se = avu.Solver.synthetic(w, rank=rank, nranks=world, generate=False, **kw)
+        barrier()
+        t0 = time.perf_counter()
+        se.set_system_ptrs(pin["vals"].data_ptr(), pin["mA"].data_ptr(), pin["mT"].data_ptr(),
+                           pin["iC"].data_ptr(), pin["b"].data_ptr())
+        se.precondition()
+        r = se.solve(x_out=xo, se_out=so, itn_limit=K, atol=0, btol=0, conlim=0, fixed_count=True)
+        barrier()
+        t_e2e = max_over_ranks(time.perf_counter() - t0)
+        h2d = sum(t.numel() * t.element_size() for t in pin.values())
+        e2e = {"value": t_e2e / K, "unit": UNIT, "h2d_bytes_per_step": int(h2d * n / K),
+               "d2h_bytes_per_step": int(2 * nloc_cols * 8 * n / K), "itn": r["itn"],
+               "note": "lsqr_set_system (pinned host A, indices, b) + lsqr_precondition + lsqr_solve(K iterations, "
+                       "fixed count) + x, se to pinned host; wall clock / K, max over ranks"}
+        se.close()
+        del pin
+        torch.cuda.synchronize()
+
+    # ---------------- device-resident timing
+    s = avu.Solver.synthetic(w, rank=rank, nranks=world, **kw)
+    t0 = time.perf_counter()
+    s.precondition()
+    s.init(itn_limit=K + Wm + 10, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=False)
+    s.sync()
+    t_setup = time.perf_counter() - t0
+    if Wm > 0:
+        s.iterate_timed(Wm)
+    barrier()
+    with ClockSampler(local) as clk:
+        r = s.iterate_timed(K)
+        barrier()
+    t_ms = max_over_ranks(r["total_ms"])
+    ap1_ms = max_over_ranks(r["aprod1_ms"] / K)
+    ap2_ms = max_over_ranks(r["aprod2_ms"] / K)
+    st, _ = s.get_state(vectors=False)
+    peak, peak_kind = measured_peaks()
+    ap1_b, ap2_b, it_b = algorithmic_bytes(w, s.n_local_rows, s.star_end - s.star_begin, s.n_shared,
+                                           s.n_local_cols)
+    if ap2_ms >= ap1_ms:
+        kname, kb, kms = "aprod2", ap2_b, ap2_ms
+    else:
+        kname, kb, kms = "aprod1", ap1_b, ap1_ms
+    achieved = kb / (kms * 1e-3) / 1e9
+    ms_step = t_ms / K
+    line = {
+        "metric": METRIC, "value": ms_step * 1e-3, "unit": UNIT, "n_gpus": n, "steps": K, "warmup": Wm,
+        "ms_per_step": ms_step, "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic",
+        "config": config_block(w, n, args, {"total_rows": w.n_obs, "setup_s": round(t_setup, 3)}),
+        "roofline": {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak,
+                     "peak_kind": f"{peak_kind} (MEASURED_PEAKS.json hbm_gbs, copy; burst)", "unit": "GB/s",
+                     "frac": round(achieved / peak, 4), "traffic": load_traffic(kname),
+                     "algorithmic_bytes_per_launch": kb, "avg_launch_ms": round(kms, 4)},
+        "iteration_roofline": {"algorithmic_bytes": it_b, "achieved_GBps": round(it_b / (ms_step * 1e-3) / 1e9, 1),
+                               "frac": round(it_b / (ms_step * 1e-3) / 1e9 / peak, 4),
+                               "aprod1_ms": round(ap1_ms, 4), "aprod2_ms": round(ap2_ms, 4),
+                               "aprod1_frac": round(ap1_b / (ap1_ms * 1e-3) / 1e9 / peak, 4),
+                               "aprod2_frac": round(ap2_b / (ap2_ms * 1e-3) / 1e9 / peak, 4)},
+        "gpu_launches": int(max_over_ranks(r["launches"])),
+        "clocks": clk.summary(),
+        "e2e": e2e,
+        "lsqr": {"itn": st["itn"], "r1norm": st["r1norm"], "arnorm": st["arnorm"]},
+    }
+    s.close()
+    if rank == 0 and n == 1 and args.cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(base, iters=args.cpu_iters)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if multi:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C2", choices=sorted(W.CONFIGS))
+    ap.add_argument("--no-e2e", dest="e2e", action="store_false")
+    ap.add_argument("--no-cpu-baseline", dest="cpu_baseline", action="store_false")
+    ap.add_argument("--cpu-iters", type=int, default=3)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -153,7 +153,9 @@ class System:
     """One rank's share (stars [star_begin, star_end)) of a generated AVU-GSR system, paper layout
     (vals[n][24], matrixIndexAstro, matrixIndexAtt, instrCol), global column numbering."""
 
-    def __init__(self, w, rank: int = 0, nranks: int = 1, generate: bool = True):
+    def __init__(self, w, rank: int = 0, nranks: int = 1, generate: bool = True, stars=None):
+        """``stars=(s0, s1)`` generates only that star range (sampled parity at full size); constraint entries
+        are then owned for those stars' astro columns and the shared columns."""
         self.w = w
         self.counts = star_counts(w)
         self.row_ptr = row_ptr(self.counts)
@@ -161,6 +163,9 @@ class System:
         self.rank, self.nranks = rank, nranks
         self.star_begin = int(self.star_begins[rank])
         self.star_end = int(self.star_begins[rank + 1])
+        if stars is not None:
+            self.star_begin, self.star_end = int(stars[0]), int(stars[1])
+            self.rank = 0
         self.row_begin = int(self.row_ptr[self.star_begin])
         self.row_end = int(self.row_ptr[self.star_end])
         n = self.n_rows = self.row_end - self.row_begin
@@ -262,10 +267,11 @@ class System:
 
 # --------------------------------------------------------------------------------------------------- O-LSQR
 def lsqr(m: int, n: int, aprod, b: np.ndarray, damp=0.0, atol=1e-8, btol=1e-8, conlim=1e8, itn_limit=None,
-         fixed_count=False, reorth=False, trace=None, want_se=True):
+         fixed_count=False, reorth=False, trace=None, want_se=True, trace_vectors=True):
     """Paige-Saunders LSQR (O-LSQR).  ``aprod`` is either a System (C products) or a python callable
     aprod(mode, vin, vout) with mode 1: vout[m] += A vin[n], mode 2: vout[n] += A^T vin[m].
-    ``trace(state_dict, u, v, w, x, var)`` is called after every iteration with COPIES of the vectors.
+    ``trace(state_dict, u, v, w, x, var)`` is called after every iteration with COPIES of the vectors
+    (``trace_vectors=False``: ``trace(state_dict)`` only, no copies -- used to time iterations).
     Returns dict(x, var, se, istop, itn, istop_first, r1norm, r2norm, anorm, acond, arnorm, xnorm, bnorm)."""
     L = lib()
     if itn_limit is None:
@@ -295,6 +301,9 @@ def lsqr(m: int, n: int, aprod, b: np.ndarray, damp=0.0, atol=1e-8, btol=1e-8, c
     if trace is not None:
         def _tr(stp, u, v, w_, xx, vv, _ctx):
             st = stp.contents.as_dict()
+            if not trace_vectors:
+                trace(st)
+                return
             arr = lambda p, k: np.ctypeslib.as_array(C.cast(p, C.POINTER(C.c_double)), (k,)).copy()
             trace(st, arr(u, m), arr(v, n), arr(w_, n), arr(xx, n), arr(vv, n))
         tcb = TRACE_FN(_tr)

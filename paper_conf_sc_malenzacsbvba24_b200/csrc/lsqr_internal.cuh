@@ -1,0 +1,103 @@
+// lsqr_internal.cuh -- device data layout and kernel launchers of liblsqr_avugsr.so (product code; shares nothing
+// with oracle/).  Layout rationale and per-kernel roofline: DESIGN.md §5-§6.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace lsqr {
+
+constexpr int kSlots = 24;           // 5 astro + 12 att + 6 instr + 1 glob
+constexpr int kThreads = 768;        // persistent row kernels: one 24-warp CTA per SM (80 regs/thread)
+constexpr int kWarpsPerCta = kThreads / 32;
+constexpr int kRedThreads = 256;     // small reduction / vector kernels
+constexpr int kInstrSmemMax = 16384; // n_instr above this -> instrumental scatter goes to L2 REDs (no smem)
+constexpr int kMaxConstr = 64;       // constraint rows handled by the one-block beta kernel
+
+// Per-row index record, 16 B: the paper's matrixIndexAtt (as k0, relative to the attitude block) and instrCol
+// (6 x u16, relative to the instrumental block) in one 128-bit word.  matrixIndexAstro is implicit: rows are
+// grouped by star (star_ptr), so the astro column is 5*star.
+struct __align__(16) IdxRec {
+  int32_t k0;
+  uint32_t ic01, ic23, ic45;  // instrCol[j] in 16-bit halves (j even: low half)
+};
+static_assert(sizeof(IdxRec) == 16, "IdxRec must be 16 bytes");
+
+// LSQR scalar state kept on the device (Paige-Saunders scalars) + control flags.
+struct DevState {
+  double alpha, beta, rhobar, phibar, anorm, acond, ddnorm, res2, xnorm, xxnorm, z, cs2, sn2, rnorm, r1norm,
+      r2norm, arnorm, bnorm;
+  double damp, atol, btol, ctol;
+  double inv_beta;   // 1/beta (1 if beta == 0): u_k = u_hat * inv_beta (u is kept unnormalised)
+  double u_scale;    // alpha_k * inv_beta_k: next aprod1 computes u_hat = A v - u_scale * u_hat
+  double inv_alpha;  // colupdate: v <- v * inv_alpha when v_pending
+  double t1, t2, t3; // x += t1 w ; w = v + t2 w ; d = t3 w
+  double rn_tmp;
+  int32_t itn, istop, istop_first, itn_limit;
+  int32_t fixed_count, halted, col_enable, v_pending, beta_pos, pad_[3];
+};
+
+// Everything a row kernel needs, passed by value.
+struct SysView {
+  const double* vals;       // [n_rows][24]
+  const IdxRec* idx;        // [n_rows]
+  const int64_t* star_ptr;  // [n_stars+1] local row offsets per local star
+  const int64_t* warp_star; // [n_warps+1] star partition of the persistent warps (balanced by rows)
+  int64_t n_rows, n_stars, n_axis, n_att, n_instr, n_sh, n_cols, A0, I0, G0;
+  int32_t n_glob, n_constr;
+  // constraint entries OWNED by this rank (S:§8(c) O-SHARD), values scaled with A
+  const double* cval;       // [n_ce]
+  const int64_t* ccol;      // [n_ce] local column
+  int64_t n_ce;
+  // aprod1 constraint dot chunks (each within one row): row, begin, end into cval/ccol
+  const int32_t* ch_row; const int64_t* ch_beg; const int64_t* ch_end; int64_t n_chunks;
+  // astro constraint entries grouped by local star (CSC by star): stars [0, n_cs)
+  int64_t n_cs; const int64_t* cs_ptr; const int32_t* cs_ak; const int64_t* cs_e;  // ak = a | (k << 8)
+  // shared-column constraint entries: shared index, constraint row, entry index
+  int64_t n_csh; const int64_t* csh_idx; const int32_t* csh_k; const int64_t* csh_e;
+};
+
+enum { AP1_LSQR = 0, AP1_PLAIN = 1 };
+enum { AP2_LSQR = 0, AP2_PLAIN = 1, AP2_COLNORM = 2 };
+
+struct GenArgs {
+  uint64_t seed;
+  int32_t b_mode;
+  double noise;
+  int64_t row_begin_global, star_begin_global;
+  int64_t n_stars_global, n_att, n_instr;
+  int32_t n_glob;
+};
+
+// ---------------------------------------------------------------------------------------------- launchers
+// All return cudaGetLastError() of the launch.
+cudaError_t launch_generate(const GenArgs& g, double* vals, IdxRec* idx, const int64_t* star_ptr, int64_t n_rows,
+                            int64_t n_stars_loc, double* b, cudaStream_t s);
+cudaError_t launch_aprod1(int mode, const SysView& S, int grid, const double* x, double* y, double* part,
+                          double* cpart, const DevState* st, cudaStream_t s);
+cudaError_t launch_aprod2(int mode, const SysView& S, int grid, const double* y, const double* ucn, double* xv,
+                          double* zsh, double* part, const DevState* st, int do_shared_constr, cudaStream_t s);
+cudaError_t launch_scale_rows(const SysView& S, int grid, double* vals, const double* D, cudaStream_t s);
+cudaError_t launch_scale_constr(const SysView& S, double* cval, const double* D, cudaStream_t s);
+// u2 partials: sum of squares of u[0..n) in a fixed grid
+cudaError_t launch_sumsq(const double* u, int64_t n, double* part, int nblk, cudaStream_t s);
+// beta kernel: reduces aprod1 partials + constraint chunks; P>1 split into pre (writes ar1) / post (reads ar1)
+cudaError_t launch_beta(int phase, const SysView& S, const double* part, int64_t n_part, const double* cpart,
+                        double* ar1, double* uc, double* ucn, const double* crhs, DevState* st, int init,
+                        cudaStream_t s);
+cudaError_t launch_cdot_add(const SysView& S, const double* cpart, const double* ar1, double* yc, cudaStream_t s);
+cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* part, int nblk, const DevState* st,
+                           cudaStream_t s);
+cudaError_t launch_add_shared(double* xsh, double* zsh, int64_t n, int mode, cudaStream_t s);
+cudaError_t launch_scalar(DevState* st, const double* part_astro, int64_t n_pa, const double* part_sh,
+                          int64_t n_ps, const double* part_wa, int64_t n_pwa, const double* part_ws, int64_t n_pws,
+                          const double* ar2_alpha2, const double* ar1_wa, int init, int32_t* host_flag,
+                          cudaStream_t s);
+cudaError_t launch_colupdate(double* v, double* w, double* x, double* var, int64_t n, int64_t A0, double* part_wa,
+                             double* part_ws, int nblk, const DevState* st, cudaStream_t s);
+cudaError_t launch_sum_to(const double* part, int64_t n, double* dst, cudaStream_t s);
+cudaError_t launch_precond_D(double* c, int64_t n, cudaStream_t s);
+cudaError_t launch_finalize(const double* x, const double* var, const double* D, int64_t n, const DevState* st,
+                            double se_t, double* x_out, double* se_out, cudaStream_t s);
+cudaError_t launch_fill(double* p, int64_t n, double v, cudaStream_t s);
+
+}  // namespace lsqr

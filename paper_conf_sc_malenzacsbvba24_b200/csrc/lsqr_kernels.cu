@@ -1,0 +1,776 @@
+// lsqr_kernels.cu -- sm_100a kernels of the AVU-GSR LSQR hot path (product code; independent of oracle/).
+//
+// Row kernels (aprod1 / aprod2 / scale) are persistent: one 1024-thread CTA per SM, every warp owns a contiguous
+// star range balanced by rows (SysView::warp_star).  A warp walks its rows 8 at a time, 4 lanes per row; lane j of
+// a row group reads the row's slots by "knot": t=0 astro j, t=1..3 attitude axis t-1 knot j, t=4 instrumental j,
+// t=5 {astro 4, instr 4, instr 5, global}[j].  Each of the 6 loads of a warp instruction reads 8 rows x 32
+// contiguous bytes, so every fetched byte of A is used; the 4 lanes of a row hit 4 consecutive attitude columns,
+// which makes the attitude gathers (aprod1) and REDs (aprod2) sector-coalesced.
+#include "lsqr_internal.cuh"
+
+namespace lsqr {
+
+// ------------------------------------------------------------------------------------------------ helpers
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+  for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+
+// fixed-order block reduction (deterministic); result valid in thread 0
+template <int NT>
+__device__ __forceinline__ double block_sum(double v) {
+  __shared__ double red_sh[NT / 32];
+  v = warp_sum(v);
+  if ((threadIdx.x & 31) == 0) red_sh[threadIdx.x >> 5] = v;
+  __syncthreads();
+  double r = 0.0;
+  if (threadIdx.x < 32) {
+    r = (threadIdx.x < NT / 32) ? red_sh[threadIdx.x] : 0.0;
+    r = warp_sum(r);
+  }
+  __syncthreads();
+  return r;
+}
+
+// ordered sum of part[0..n) by one block (thread t sums t, t+NT, ...), result in thread 0
+template <int NT>
+__device__ __forceinline__ double ordered_sum(const double* __restrict__ part, int64_t n) {
+  double s = 0.0;
+  for (int64_t i = threadIdx.x; i < n; i += NT) s += part[i];
+  return block_sum<NT>(s);
+}
+
+__device__ __forceinline__ uint32_t ic_of(const IdxRec& r, int q) {  // instrCol q (0..5), relative to I0
+  uint32_t w = q < 2 ? r.ic01 : (q < 4 ? r.ic23 : r.ic45);
+  return (w >> ((q & 1) * 16)) & 0xffffu;
+}
+
+__device__ __forceinline__ int slot_of(int t, int j) {
+  return t == 0 ? j : (t <= 3 ? 5 + 4 * (t - 1) + j : (t == 4 ? 17 + j : (j == 0 ? 4 : 20 + j)));
+}
+
+// ------------------------------------------------------------------------------------------------ generator
+// O-GEN (docs/GENERATOR.md): splitmix64-based counter hash; integer-only, exact int->double conversions, so the
+// device arrays are bit-identical to any other implementation of the spec.
+__device__ __forceinline__ uint64_t g_mix(uint64_t z) {
+  z += 0x9E3779B97F4A7C15ULL;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ULL;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBULL;
+  return z ^ (z >> 31);
+}
+__device__ __forceinline__ uint64_t g_hash(uint64_t seed, uint64_t tag, uint64_t i, uint64_t j) {
+  return g_mix(g_mix(g_mix(seed ^ (tag << 56)) ^ i) ^ j);
+}
+__device__ __forceinline__ double g_pm1(uint64_t h) {
+  return __dmul_rn(__ll2double_rn((long long)(h >> 10) - (1LL << 53)), 0x1p-53);
+}
+
+__global__ void k_generate(GenArgs g, double* __restrict__ vals, IdxRec* __restrict__ idx,
+                           const int64_t* __restrict__ star_ptr, int64_t n_rows, int64_t n_stars_loc,
+                           double* __restrict__ b) {
+  const int64_t n_axis = g.n_att / 3, grp = g.n_instr / 6;
+  const int64_t A0g = 5 * g.n_stars_global, I0g = A0g + g.n_att, G0g = I0g + g.n_instr;
+  for (int64_t li = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; li < n_rows;
+       li += (int64_t)gridDim.x * blockDim.x) {
+    // local star: largest s with star_ptr[s] <= li
+    int64_t lo = 0, hi = n_stars_loc;  // invariant star_ptr[lo] <= li < star_ptr[hi]
+    while (hi - lo > 1) {
+      int64_t mid = (lo + hi) >> 1;
+      if (star_ptr[mid] <= li) lo = mid; else hi = mid;
+    }
+    const uint64_t i = (uint64_t)(g.row_begin_global + li);
+    const int64_t gstar = g.star_begin_global + lo;
+    const int64_t k0 = (int64_t)(g_hash(g.seed, 2, i, 0) % (uint64_t)(n_axis - 3));
+    uint32_t ic[6];
+#pragma unroll
+    for (int j = 0; j < 6; ++j) ic[j] = (uint32_t)(j * grp + (int64_t)(g_hash(g.seed, 3, i, j) % (uint64_t)grp));
+    IdxRec rec;
+    rec.k0 = (int32_t)k0;
+    rec.ic01 = ic[0] | (ic[1] << 16);
+    rec.ic23 = ic[2] | (ic[3] << 16);
+    rec.ic45 = ic[4] | (ic[5] << 16);
+    idx[li] = rec;
+    double v[kSlots];
+#pragma unroll
+    for (int s = 0; s < kSlots; ++s) v[s] = g_pm1(g_hash(g.seed, 4, i, s));
+    if (g.n_glob == 0) v[23] = 0.0;
+    double* rp = vals + li * kSlots;
+#pragma unroll
+    for (int s = 0; s < kSlots; s += 2) *reinterpret_cast<double2*>(rp + s) = make_double2(v[s], v[s + 1]);
+    if (g.b_mode == 0) {
+      b[li] = g_pm1(g_hash(g.seed, 5, i, 0));
+    } else {  // planted: b = sum_s val_s * x_true[col_s] in slot order, every op rounded (no FMA), + noise term
+      double acc = 0.0;
+#pragma unroll
+      for (int s = 0; s < kSlots; ++s) {
+        if (s == 23 && g.n_glob == 0) continue;
+        int64_t col = s < 5 ? 5 * gstar + s
+                            : (s < 17 ? A0g + ((s - 5) / 4) * n_axis + k0 + ((s - 5) % 4)
+                                      : (s < 23 ? I0g + ic[s - 17] : G0g));
+        acc = __dadd_rn(acc, __dmul_rn(v[s], g_pm1(g_hash(g.seed, 7, (uint64_t)col, 0))));
+      }
+      b[li] = __dadd_rn(acc, __dmul_rn(g.noise, g_pm1(g_hash(g.seed, 6, i, 0))));
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------ row loading
+struct RowRaw {
+  double v[6];
+  IdxRec rec;
+  double y;   // u_hat (LSQR) or y (plain) of the row
+};
+
+__device__ __forceinline__ void load_row(const SysView& S, const double* __restrict__ yv, int64_t row, bool valid,
+                                         int j, RowRaw& o) {
+  if (valid) {
+    const double* rp = S.vals + row * kSlots;
+#pragma unroll
+    for (int t = 0; t < 6; ++t) o.v[t] = __ldg(rp + slot_of(t, j));
+    const int4 q = __ldg(reinterpret_cast<const int4*>(S.idx) + row);  // 16 B, broadcast within the row group
+    o.rec.k0 = q.x;
+    o.rec.ic01 = (uint32_t)q.y; o.rec.ic23 = (uint32_t)q.z; o.rec.ic45 = (uint32_t)q.w;
+    o.y = yv ? __ldg(yv + row) : 0.0;
+  } else {
+#pragma unroll
+    for (int t = 0; t < 6; ++t) o.v[t] = 0.0;
+    o.rec.k0 = 0; o.rec.ic01 = o.rec.ic23 = o.rec.ic45 = 0;
+    o.y = 0.0;
+  }
+}
+
+// local column of the lane's slot t (t=5, j=3 is the global column; caller masks it when n_glob == 0)
+__device__ __forceinline__ int64_t col_of(const SysView& S, int t, int j, int64_t star, const IdxRec& r) {
+  if (t == 0) return 5 * star + j;
+  if (t <= 3) return S.A0 + (int64_t)(t - 1) * S.n_axis + r.k0 + j;
+  if (t == 4) return S.I0 + ic_of(r, j);
+  return j == 0 ? 5 * star + 4 : (j == 3 ? S.G0 : S.I0 + ic_of(r, 3 + j));
+}
+
+// ------------------------------------------------------------------------------------------------ aprod1
+// MODE AP1_LSQR:  u_hat[i] = sum_s a_is v[col_is] - u_scale * u_hat[i];  per-warp partial of u_hat^2 (beta^2).
+// MODE AP1_PLAIN: y[i] += sum_s a_is x[col_is].
+// Constraint rows: per-chunk partial dots of the owned entries -> cpart (combined by k_beta / k_cdot).
+template <int MODE>
+__global__ void __launch_bounds__(kThreads, 1)
+    k_aprod1(SysView S, const double* __restrict__ x, double* __restrict__ y, double* __restrict__ part,
+             double* __restrict__ cpart, const DevState* __restrict__ st) {
+  if (MODE == AP1_LSQR && st->halted) return;
+  const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const double uscale = MODE == AP1_LSQR ? st->u_scale : 0.0;
+  const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
+  const int64_t r_lo = S.star_ptr[s_lo], r_hi = S.star_ptr[s_hi];
+  const bool glob_ok = S.n_glob != 0;
+  int64_t s = s_lo;
+  double b2 = 0.0;
+  RowRaw cur, nxt;
+  load_row(S, y, r_lo + r, r_lo + r < r_hi, j, cur);
+  for (int64_t base = r_lo; base < r_hi; base += 8) {
+    const int64_t row = base + r;
+    const bool valid = row < r_hi;
+    const int64_t nrow = row + 8;
+    load_row(S, y, nrow, nrow < r_hi, j, nxt);  // prefetch next row group
+    double p = 0.0;
+    if (valid) {
+      while (S.star_ptr[s + 1] <= row) ++s;
+#pragma unroll
+      for (int t = 0; t < 6; ++t) {
+        const int64_t c = col_of(S, t, j, s, cur.rec);
+        const double xv = (t == 5 && j == 3 && !glob_ok) ? 0.0 : __ldg(x + c);
+        p = fma(cur.v[t], xv, p);
+      }
+    }
+    p += __shfl_xor_sync(0xffffffffu, p, 1);
+    p += __shfl_xor_sync(0xffffffffu, p, 2);
+    if (valid && j == 0) {
+      if (MODE == AP1_LSQR) {
+        const double un = p - uscale * cur.y;
+        y[row] = un;
+        b2 = fma(un, un, b2);
+      } else {
+        y[row] = cur.y + p;
+      }
+    }
+    cur = nxt;
+  }
+  if (MODE == AP1_LSQR) {
+    b2 = warp_sum(b2);
+    if (lane == 0) part[gw] = b2;
+  }
+  // constraint rows: owned-entry partial dots, chunk by chunk
+  for (int64_t c = gw; c < S.n_chunks; c += W) {
+    double acc = 0.0;
+    for (int64_t e = S.ch_beg[c] + lane; e < S.ch_end[c]; e += 32) acc = fma(S.cval[e], __ldg(x + S.ccol[e]), acc);
+    acc = warp_sum(acc);
+    if (lane == 0) cpart[c] = acc;
+  }
+}
+
+// ------------------------------------------------------------------------------------------------ aprod2
+// z = A^T y, scatter-free on the astrometric block (one warp owns whole stars, so the 5 astro sums of a star are
+// a warp reduction), hierarchical on the shared slice: attitude -> sector-coalesced FP64 REDs into
+// the L2-resident z_sh (P:L427-434 uses atomics), instrumental -> CTA-private shared-memory accumulator flushed
+// once per CTA, global -> register + warp shuffle, one RED per warp.
+//   MODE AP2_LSQR:    y = u_hat * inv_beta; astro: v[c] = z + constr - beta v[c] (v' of Paige-Saunders, unnormalised),
+//                     per-warp partial of v'^2 (alpha^2, astro part).  Shared slice left in zsh (vshared finishes).
+//   MODE AP2_PLAIN:   astro: x[c] += z (+ constraint entries with y_c); shared slice accumulated in zsh.
+//   MODE AP2_COLNORM: contributions a^2 (column sums of squares, O-PREC); astro: c[c] = z; shared in zsh.
+template <int MODE, bool SMEM_INSTR>
+__global__ void __launch_bounds__(kThreads, 1)
+    k_aprod2(SysView S, const double* __restrict__ yv, const double* __restrict__ ucn, double* __restrict__ xv,
+             double* __restrict__ zsh, double* __restrict__ part, const DevState* __restrict__ st,
+             int do_shared_constr) {
+  extern __shared__ double sh_instr[];
+  if (MODE == AP2_LSQR && (st->halted || !st->beta_pos)) return;
+  if (SMEM_INSTR) {
+    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_instr[i] = 0.0;
+    __syncthreads();
+  }
+  const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const double inv_beta = MODE == AP2_LSQR ? st->inv_beta : 1.0;
+  const double beta = MODE == AP2_LSQR ? st->beta : 0.0;
+  const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
+  const int64_t r_lo = S.star_ptr[s_lo], r_hi = S.star_ptr[s_hi];
+  const bool glob_ok = S.n_glob != 0;
+  double* z_att = zsh;
+  double* z_ins = SMEM_INSTR ? sh_instr : zsh + S.n_att;
+  double gacc = 0.0, a2 = 0.0, acc0 = 0.0, acc1 = 0.0;
+  int64_t s = s_lo;      // lane-local star of the lane's row
+  int64_t cs = s_lo;     // warp-uniform star being accumulated
+  int64_t cs_end = (cs < s_hi) ? S.star_ptr[cs + 1] : 0;
+
+  auto finalize = [&](int64_t star) {
+    double z0 = acc0, z1 = acc1;
+    z0 += __shfl_xor_sync(0xffffffffu, z0, 4);
+    z0 += __shfl_xor_sync(0xffffffffu, z0, 8);
+    z0 += __shfl_xor_sync(0xffffffffu, z0, 16);
+    z1 += __shfl_xor_sync(0xffffffffu, z1, 4);
+    z1 += __shfl_xor_sync(0xffffffffu, z1, 8);
+    z1 += __shfl_xor_sync(0xffffffffu, z1, 16);
+    if (lane < 4) {
+      if (star < S.n_cs) {  // constraint entries on this star's astro columns (after all rows, as O-AP2)
+        for (int64_t e = S.cs_ptr[star]; e < S.cs_ptr[star + 1]; ++e) {
+          const int ak = S.cs_ak[e], a = ak & 0xff, k = ak >> 8;
+          const double cv = S.cval[S.cs_e[e]];
+          const double c = MODE == AP2_COLNORM ? cv * cv : cv * ucn[k];
+          if (a == j) z0 += c;
+          if (j == 0 && a == 4) z1 += c;
+        }
+      }
+      const int64_t c0 = 5 * star + j;
+      if (MODE == AP2_LSQR) {
+        const double vn = z0 - beta * xv[c0];
+        xv[c0] = vn;
+        a2 = fma(vn, vn, a2);
+        if (j == 0) {
+          const double vn1 = z1 - beta * xv[5 * star + 4];
+          xv[5 * star + 4] = vn1;
+          a2 = fma(vn1, vn1, a2);
+        }
+      } else if (MODE == AP2_PLAIN) {
+        xv[c0] += z0;
+        if (j == 0) xv[5 * star + 4] += z1;
+      } else {
+        xv[c0] = z0;
+        if (j == 0) xv[5 * star + 4] = z1;
+      }
+    }
+  };
+
+  RowRaw cur, nxt;
+  const double* ysrc = MODE == AP2_COLNORM ? nullptr : yv;
+  load_row(S, ysrc, r_lo + r, r_lo + r < r_hi, j, cur);
+  for (int64_t base = r_lo; base < r_hi; base += 8) {
+    const int64_t row = base + r;
+    const bool valid = row < r_hi;
+    const int64_t nrow = row + 8;
+    load_row(S, ysrc, nrow, nrow < r_hi, j, nxt);
+    double c[6];
+    const double yr = MODE == AP2_LSQR ? cur.y * inv_beta : cur.y;
+#pragma unroll
+    for (int t = 0; t < 6; ++t) c[t] = MODE == AP2_COLNORM ? cur.v[t] * cur.v[t] : cur.v[t] * yr;
+    if (valid) {
+      while (S.star_ptr[s + 1] <= row) ++s;
+      // attitude: 3 axes x 4 consecutive knots -> sector-coalesced REDs (one per axis per lane)
+#pragma unroll
+      for (int t = 1; t <= 3; ++t) atomicAdd(z_att + (int64_t)(t - 1) * S.n_axis + cur.rec.k0 + j, c[t]);
+      // instrumental
+      atomicAdd(z_ins + ic_of(cur.rec, j), c[4]);
+      if (j == 1 || j == 2) atomicAdd(z_ins + ic_of(cur.rec, 3 + j), c[5]);
+      if (j == 3 && glob_ok) gacc += c[5];
+    }
+    // astrometric: segmented by star (rows are grouped by star)
+    const double c0 = c[0], c5 = (j == 0) ? c[5] : 0.0;
+    const int64_t step_end = base + 8 < r_hi ? base + 8 : r_hi;
+    while (true) {
+      if (valid && s == cs) { acc0 += c0; acc1 += c5; }
+      if (cs < s_hi && cs_end <= step_end) {
+        finalize(cs);
+        acc0 = 0.0; acc1 = 0.0;
+        ++cs;
+        if (cs >= s_hi) break;
+        cs_end = S.star_ptr[cs + 1];
+      } else {
+        break;
+      }
+    }
+    cur = nxt;
+  }
+  while (cs < s_hi) {  // empty trailing stars
+    acc0 = 0.0; acc1 = 0.0;
+    finalize(cs);
+    ++cs;
+  }
+  // global column: one RED per warp
+  if (glob_ok) {
+    gacc = warp_sum(gacc);
+    if (lane == 0 && gacc != 0.0) atomicAdd(zsh + S.n_att + S.n_instr, gacc);
+  }
+  if (MODE == AP2_LSQR) {
+    a2 = warp_sum(a2);
+    if (lane == 0) part[gw] = a2;
+  }
+  // constraint entries on shared columns (owned by rank 0 only; the host passes n_csh = 0 elsewhere)
+  if (do_shared_constr) {
+    for (int64_t e = gw * 32 + lane; e < S.n_csh; e += W * 32) {
+      const double cv = S.cval[S.csh_e[e]];
+      const double c = MODE == AP2_COLNORM ? cv * cv : cv * ucn[S.csh_k[e]];
+      atomicAdd(zsh + S.csh_idx[e], c);
+    }
+  }
+  if (SMEM_INSTR) {
+    __syncthreads();
+    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
+      const double v = sh_instr[i];
+      if (v != 0.0) atomicAdd(zsh + S.n_att + i, v);
+    }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------ scale rows (O-PREC)
+__global__ void __launch_bounds__(kThreads, 1)
+    k_scale_rows(SysView S, double* __restrict__ vals, const double* __restrict__ D) {
+  const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
+  const int64_t r_lo = S.star_ptr[s_lo], r_hi = S.star_ptr[s_hi];
+  int64_t s = s_lo;
+  for (int64_t base = r_lo; base < r_hi; base += 8) {
+    const int64_t row = base + r;
+    if (row >= r_hi) continue;
+    while (S.star_ptr[s + 1] <= row) ++s;
+    const IdxRec rec = S.idx[row];
+    double* rp = vals + row * kSlots;
+#pragma unroll
+    for (int t = 0; t < 6; ++t) {
+      if (t == 5 && j == 3 && S.n_glob == 0) continue;
+      const int sl = slot_of(t, j);
+      rp[sl] = rp[sl] * D[col_of(S, t, j, s, rec)];
+    }
+  }
+}
+
+__global__ void k_scale_constr(SysView S, double* __restrict__ cval, const double* __restrict__ D) {
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < S.n_ce; e += (int64_t)gridDim.x * blockDim.x)
+    cval[e] = cval[e] * D[S.ccol[e]];
+}
+
+// ------------------------------------------------------------------------------------------------ vectors
+__global__ void __launch_bounds__(kRedThreads) k_sumsq(const double* __restrict__ u, int64_t n,
+                                                       double* __restrict__ part) {
+  double s = 0.0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    s = fma(u[i], u[i], s);
+  s = block_sum<kRedThreads>(s);
+  if (threadIdx.x == 0) part[blockIdx.x] = s;
+}
+
+// phase 0: single rank (reduce + finish); 1: multi-rank pre-AR1 (write ar1); 2: multi-rank post-AR1 (finish);
+// 3: plain aprod1 constraint dots into ar1 (no state); init: u_hat = b (beta_0 = ||b||, O-1).
+__global__ void __launch_bounds__(kRedThreads)
+    k_beta(int phase, SysView S, const double* __restrict__ part, int64_t n_part, const double* __restrict__ cpart,
+           double* __restrict__ ar1, double* __restrict__ uc, double* __restrict__ ucn,
+           const double* __restrict__ crhs, DevState* __restrict__ st, int init) {
+  __shared__ double cdot_sh[64];
+  __shared__ double b2_sh;
+  if (phase != 3 && !init && st->halted) return;
+  const int nc = S.n_constr;
+  if (phase != 2) {
+    const double b2 = phase == 3 ? 0.0 : ordered_sum<kRedThreads>(part, n_part);
+    if (threadIdx.x == 0) b2_sh = b2;
+    // chunk partials -> per-row dots (chunks are in row order; each row's chunks summed in order)
+    if (threadIdx.x < nc) {
+      double d = 0.0;
+      if (!init)
+        for (int64_t c = 0; c < S.n_chunks; ++c)
+          if (S.ch_row[c] == (int)threadIdx.x) d += cpart[c];
+      cdot_sh[threadIdx.x] = d;
+    }
+    __syncthreads();
+    if (phase == 1 || phase == 3) {
+      if (threadIdx.x < nc) ar1[threadIdx.x] = cdot_sh[threadIdx.x];
+      if (threadIdx.x == 0 && phase == 1) ar1[nc] = b2_sh;
+      return;
+    }
+  } else {
+    if (threadIdx.x < nc) cdot_sh[threadIdx.x] = ar1[threadIdx.x];
+    if (threadIdx.x == 0) b2_sh = ar1[nc];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    const double us = st->u_scale;
+    double b2 = b2_sh;
+    for (int k = 0; k < nc; ++k) {
+      const double un = init ? (crhs ? crhs[k] : 0.0) : cdot_sh[k] - us * uc[k];
+      uc[k] = un;
+      b2 = fma(un, un, b2);
+    }
+    const double beta = sqrt(b2);
+    const int pos = beta > 0.0;
+    const double ib = pos ? 1.0 / beta : 1.0;
+    if (init) {
+      st->bnorm = beta;
+    } else if (pos) {
+      const double a = st->alpha, d = st->damp;
+      st->anorm = sqrt(st->anorm * st->anorm + a * a + beta * beta + d * d);
+    }
+    st->beta = beta;
+    st->beta_pos = pos;
+    st->inv_beta = ib;
+    for (int k = 0; k < nc; ++k) ucn[k] = uc[k] * ib;
+  }
+}
+
+// plain aprod1: y_c[k] += cdot[k] (cdot from chunks, or already allreduced in ar1 when from_ar1)
+__global__ void k_cdot_add(SysView S, const double* __restrict__ cpart, const double* __restrict__ ar1,
+                           double* __restrict__ yc) {
+  const int k = threadIdx.x;
+  if (k >= S.n_constr) return;
+  double d = 0.0;
+  if (ar1) d = ar1[k];
+  else
+    for (int64_t c = 0; c < S.n_chunks; ++c)
+      if (S.ch_row[c] == k) d += cpart[c];
+  yc[k] += d;
+}
+
+__global__ void __launch_bounds__(kRedThreads)
+    k_vshared(int64_t n_sh, double* __restrict__ vsh, double* __restrict__ zsh, double* __restrict__ part,
+              const DevState* __restrict__ st) {
+  if (st->halted || !st->beta_pos) return;
+  const double beta = st->beta;
+  double a2 = 0.0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_sh; i += (int64_t)gridDim.x * blockDim.x) {
+    const double vn = zsh[i] - beta * vsh[i];
+    vsh[i] = vn;
+    zsh[i] = 0.0;
+    a2 = fma(vn, vn, a2);
+  }
+  a2 = block_sum<kRedThreads>(a2);
+  if (threadIdx.x == 0) part[blockIdx.x] = a2;
+}
+
+// mode 0: x += z, z = 0 (plain aprod2);  mode 1: x = z, z = 0 (column norms)
+__global__ void k_add_shared(double* __restrict__ xsh, double* __restrict__ zsh, int64_t n, int mode) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    xsh[i] = mode == 0 ? xsh[i] + zsh[i] : zsh[i];
+    zsh[i] = 0.0;
+  }
+}
+
+// O-3 steps c-j (rotation, norm estimates, stopping tests) in one thread; Paige & Saunders (lsqr.f form).
+__global__ void __launch_bounds__(kRedThreads)
+    k_scalar(DevState* __restrict__ st, const double* __restrict__ part_astro, int64_t n_pa,
+             const double* __restrict__ part_sh, int64_t n_ps, const double* __restrict__ part_wa, int64_t n_pwa,
+             const double* __restrict__ part_ws, int64_t n_pws, const double* __restrict__ ar2_alpha2,
+             const double* __restrict__ ar1_wa, int init, int32_t* __restrict__ host_flag) {
+  if (!init && st->halted) {
+    if (threadIdx.x == 0) st->col_enable = 0;
+    return;
+  }
+  const int bp = st->beta_pos;
+  // alpha^2 = ||v'||^2: astro part (per-warp partials of aprod2, or the allreduced value on several ranks)
+  // + shared part (replicated, counted once).  ||w||^2 likewise (for ddnorm).
+  double a2 = 0.0;
+  if (bp) {
+    a2 = ar2_alpha2 ? 0.0 : ordered_sum<kRedThreads>(part_astro, n_pa);
+    a2 += ordered_sum<kRedThreads>(part_sh, n_ps);
+  }
+  double w2 = 0.0;
+  if (!init) {
+    w2 = ar1_wa ? 0.0 : ordered_sum<kRedThreads>(part_wa, n_pwa);
+    w2 += ordered_sum<kRedThreads>(part_ws, n_pws);
+  }
+  if (threadIdx.x != 0) return;
+  if (bp && ar2_alpha2) a2 += *ar2_alpha2;
+  if (!init && ar1_wa) w2 += *ar1_wa;
+  const double eps = 0x1p-52;
+  if (init) {
+    const double alpha = bp ? sqrt(a2) : 0.0;
+    const double beta = st->beta;
+    st->alpha = alpha;
+    st->inv_alpha = alpha > 0.0 ? 1.0 / alpha : 1.0;
+    st->v_pending = bp;
+    st->rhobar = alpha; st->phibar = beta; st->rnorm = beta; st->r1norm = beta; st->r2norm = beta;
+    st->anorm = 0; st->acond = 0; st->ddnorm = 0; st->res2 = 0; st->xnorm = 0; st->xxnorm = 0; st->z = 0;
+    st->cs2 = -1.0; st->sn2 = 0.0;
+    st->arnorm = alpha * beta;
+    st->t1 = 0.0; st->t2 = 0.0; st->t3 = 0.0;
+    st->col_enable = 1;
+    st->itn = 0; st->istop = 0; st->istop_first = 0;
+    st->halted = (alpha * beta == 0.0) ? 1 : 0;
+    st->u_scale = alpha * st->inv_beta;
+  } else {
+    st->itn += 1;
+    double alpha = st->alpha;
+    if (bp) {
+      alpha = sqrt(a2);
+      st->inv_alpha = alpha > 0.0 ? 1.0 / alpha : 1.0;
+      st->v_pending = 1;
+    } else {
+      st->v_pending = 0;
+    }
+    st->alpha = alpha;
+    const double beta = st->beta, damp = st->damp, dampsq = damp * damp;
+    double rhobar = st->rhobar, phibar = st->phibar, psi, rhobar1;
+    if (damp > 0.0) {  // c.
+      rhobar1 = sqrt(rhobar * rhobar + dampsq);
+      const double cs1 = rhobar / rhobar1, sn1 = damp / rhobar1;
+      psi = sn1 * phibar;
+      phibar = cs1 * phibar;
+    } else {
+      rhobar1 = rhobar;
+      psi = 0.0;
+    }
+    const double rho = sqrt(rhobar1 * rhobar1 + beta * beta);  // d.
+    const double cs = rhobar1 / rho, sn = beta / rho;
+    const double theta = sn * alpha;
+    rhobar = -cs * alpha;
+    const double phi = cs * phibar;
+    phibar = sn * phibar;
+    const double tau = sn * phi;
+    const double t1 = phi / rho, t2 = -theta / rho, t3 = 1.0 / rho;  // e. (applied by k_colupdate)
+    st->t1 = t1; st->t2 = t2; st->t3 = t3;
+    const double ddnorm = st->ddnorm + t3 * t3 * w2;  // sum_j (t3 w_j)^2 with w the pre-update w
+    // f.
+    const double delta = st->sn2 * rho, gambar = -st->cs2 * rho, rhs = phi - delta * st->z, zbar = rhs / gambar;
+    const double xnorm = sqrt(st->xxnorm + zbar * zbar);
+    const double gamma = sqrt(gambar * gambar + theta * theta);
+    st->cs2 = gambar / gamma;
+    st->sn2 = theta / gamma;
+    st->z = rhs / gamma;
+    st->xxnorm = st->xxnorm + st->z * st->z;
+    // g.
+    const double anorm = st->anorm;
+    const double acond = anorm * sqrt(ddnorm);
+    const double res2 = st->res2 + psi * psi;
+    const double rnorm = sqrt(phibar * phibar + res2);
+    const double arnorm = alpha * fabs(tau);
+    double r1norm;
+    if (damp > 0.0) {
+      const double r1sq = rnorm * rnorm - dampsq * st->xxnorm;
+      r1norm = sqrt(fabs(r1sq));
+      if (r1sq < 0) r1norm = -r1norm;
+    } else {
+      r1norm = rnorm;
+    }
+    // h.
+    const double bnorm = st->bnorm;
+    const double test1 = rnorm / bnorm, test2 = arnorm / (anorm * rnorm + eps), test3 = 1.0 / (acond + eps);
+    const double tt1 = test1 / (1.0 + anorm * xnorm / bnorm);
+    const double rtol = st->btol + st->atol * anorm * xnorm / bnorm;
+    // i.
+    int is = 0;
+    if (st->itn >= st->itn_limit) is = 7;
+    if (1.0 + test3 <= 1.0) is = 6;
+    if (1.0 + test2 <= 1.0) is = 5;
+    if (1.0 + tt1 <= 1.0) is = 4;
+    if (test3 <= st->ctol) is = 3;
+    if (test2 <= st->atol) is = 2;
+    if (test1 <= rtol) is = 1;
+    st->rhobar = rhobar; st->phibar = phibar; st->ddnorm = ddnorm; st->xnorm = xnorm; st->acond = acond;
+    st->res2 = res2; st->rnorm = rnorm; st->r1norm = r1norm; st->r2norm = rnorm; st->arnorm = arnorm;
+    st->istop = is;
+    if (is != 0 && st->istop_first == 0) st->istop_first = is;
+    st->col_enable = 1;
+    st->u_scale = alpha * st->inv_beta;
+    if ((is != 0 && !st->fixed_count) || st->itn >= st->itn_limit) st->halted = 1;
+  }
+  if (host_flag) *reinterpret_cast<volatile int32_t*>(host_flag) = st->halted | (st->itn << 1);
+}
+
+// O-3e: v <- v/alpha (if pending); d = t3 w; var += d^2; x += t1 w; w = v + t2 w;  partials of ||w_new||^2 split
+// into the local astro columns (i < A0) and the replicated shared slice (i >= A0).
+__global__ void __launch_bounds__(kRedThreads)
+    k_colupdate(double* __restrict__ v, double* __restrict__ w, double* __restrict__ x, double* __restrict__ var,
+                int64_t n, int64_t A0, double* __restrict__ part_wa, double* __restrict__ part_ws,
+                const DevState* __restrict__ st) {
+  if (!st->col_enable) return;
+  const double ia = st->v_pending ? st->inv_alpha : 1.0;
+  const double t1 = st->t1, t2 = st->t2, t3 = st->t3;
+  double wa = 0.0, ws = 0.0;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const double vi = v[i] * ia, wi = w[i];
+    const double d = t3 * wi;
+    var[i] = fma(d, d, var[i]);
+    x[i] = fma(t1, wi, x[i]);
+    const double wnew = fma(t2, wi, vi);
+    w[i] = wnew;
+    v[i] = vi;
+    if (i < A0) wa = fma(wnew, wnew, wa);
+    else ws = fma(wnew, wnew, ws);
+  }
+  wa = block_sum<kRedThreads>(wa);
+  ws = block_sum<kRedThreads>(ws);
+  if (threadIdx.x == 0) {
+    part_wa[blockIdx.x] = wa;
+    part_ws[blockIdx.x] = ws;
+  }
+}
+
+__global__ void k_sum_to(const double* __restrict__ part, int64_t n, double* __restrict__ dst) {
+  const double s = ordered_sum<kRedThreads>(part, n);
+  if (threadIdx.x == 0) *dst = s;
+}
+
+__global__ void k_precond_D(double* __restrict__ c, int64_t n) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    c[i] = c[i] > 0.0 ? 1.0 / sqrt(c[i]) : 1.0;
+}
+
+// O-4/O-5: se_j = D_j * s * sqrt(var_j), x_j = D_j * x_j,  s = r2norm / sqrt(t)
+__global__ void k_finalize(const double* __restrict__ x, const double* __restrict__ var, const double* __restrict__ D,
+                           int64_t n, const DevState* __restrict__ st, double se_t, double* __restrict__ xo,
+                           double* __restrict__ so) {
+  const double s = st->r2norm / sqrt(se_t);
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    if (xo) xo[i] = D[i] * x[i];
+    if (so) so[i] = D[i] * (s * sqrt(var[i]));
+  }
+}
+
+__global__ void k_fill(double* __restrict__ p, int64_t n, double v) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    p[i] = v;
+}
+
+// ------------------------------------------------------------------------------------------------ launchers
+static int vec_grid(int64_t n, int maxb) {
+  int64_t b = (n + kRedThreads - 1) / kRedThreads;
+  if (b < 1) b = 1;
+  return (int)(b < maxb ? b : maxb);
+}
+
+cudaError_t launch_generate(const GenArgs& g, double* vals, IdxRec* idx, const int64_t* star_ptr, int64_t n_rows,
+                            int64_t n_stars_loc, double* b, cudaStream_t s) {
+  if (n_rows == 0) return cudaSuccess;
+  k_generate<<<vec_grid(n_rows, 148 * 16), kRedThreads, 0, s>>>(g, vals, idx, star_ptr, n_rows, n_stars_loc, b);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_aprod1(int mode, const SysView& S, int grid, const double* x, double* y, double* part,
+                          double* cpart, const DevState* st, cudaStream_t s) {
+  if (mode == AP1_LSQR) k_aprod1<AP1_LSQR><<<grid, kThreads, 0, s>>>(S, x, y, part, cpart, st);
+  else k_aprod1<AP1_PLAIN><<<grid, kThreads, 0, s>>>(S, x, y, part, cpart, st);
+  return cudaGetLastError();
+}
+
+template <int MODE, bool SM>
+static cudaError_t ap2(const SysView& S, int grid, const double* y, const double* ucn, double* xv, double* zsh,
+                       double* part, const DevState* st, int dsc, cudaStream_t s) {
+  size_t smem = SM ? (size_t)S.n_instr * sizeof(double) : 0;
+  static bool attr_set = false;
+  if (SM && !attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(k_aprod2<MODE, SM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)(kInstrSmemMax * sizeof(double)));
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  k_aprod2<MODE, SM><<<grid, kThreads, smem, s>>>(S, y, ucn, xv, zsh, part, st, dsc);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_aprod2(int mode, const SysView& S, int grid, const double* y, const double* ucn, double* xv,
+                          double* zsh, double* part, const DevState* st, int dsc, cudaStream_t s) {
+  const bool sm = S.n_instr <= kInstrSmemMax;
+  switch (mode) {
+    case AP2_LSQR: return sm ? ap2<AP2_LSQR, true>(S, grid, y, ucn, xv, zsh, part, st, dsc, s)
+                             : ap2<AP2_LSQR, false>(S, grid, y, ucn, xv, zsh, part, st, dsc, s);
+    case AP2_PLAIN: return sm ? ap2<AP2_PLAIN, true>(S, grid, y, ucn, xv, zsh, part, st, dsc, s)
+                              : ap2<AP2_PLAIN, false>(S, grid, y, ucn, xv, zsh, part, st, dsc, s);
+    default: return sm ? ap2<AP2_COLNORM, true>(S, grid, y, ucn, xv, zsh, part, st, dsc, s)
+                       : ap2<AP2_COLNORM, false>(S, grid, y, ucn, xv, zsh, part, st, dsc, s);
+  }
+}
+
+cudaError_t launch_scale_rows(const SysView& S, int grid, double* vals, const double* D, cudaStream_t s) {
+  k_scale_rows<<<grid, kThreads, 0, s>>>(S, vals, D);
+  return cudaGetLastError();
+}
+cudaError_t launch_scale_constr(const SysView& S, double* cval, const double* D, cudaStream_t s) {
+  if (S.n_ce == 0) return cudaSuccess;
+  k_scale_constr<<<vec_grid(S.n_ce, 148), kRedThreads, 0, s>>>(S, cval, D);
+  return cudaGetLastError();
+}
+cudaError_t launch_sumsq(const double* u, int64_t n, double* part, int nblk, cudaStream_t s) {
+  k_sumsq<<<nblk, kRedThreads, 0, s>>>(u, n, part);
+  return cudaGetLastError();
+}
+cudaError_t launch_beta(int phase, const SysView& S, const double* part, int64_t n_part, const double* cpart,
+                        double* ar1, double* uc, double* ucn, const double* crhs, DevState* st, int init,
+                        cudaStream_t s) {
+  k_beta<<<1, kRedThreads, 0, s>>>(phase, S, part, n_part, cpart, ar1, uc, ucn, crhs, st, init);
+  return cudaGetLastError();
+}
+cudaError_t launch_cdot_add(const SysView& S, const double* cpart, const double* ar1, double* yc, cudaStream_t s) {
+  if (S.n_constr == 0) return cudaSuccess;
+  k_cdot_add<<<1, 64, 0, s>>>(S, cpart, ar1, yc);
+  return cudaGetLastError();
+}
+cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* part, int nblk, const DevState* st,
+                           cudaStream_t s) {
+  k_vshared<<<nblk, kRedThreads, 0, s>>>(S.n_sh, vsh, zsh, part, st);
+  return cudaGetLastError();
+}
+cudaError_t launch_add_shared(double* xsh, double* zsh, int64_t n, int mode, cudaStream_t s) {
+  k_add_shared<<<vec_grid(n, 148 * 4), kRedThreads, 0, s>>>(xsh, zsh, n, mode);
+  return cudaGetLastError();
+}
+cudaError_t launch_scalar(DevState* st, const double* part_astro, int64_t n_pa, const double* part_sh,
+                          int64_t n_ps, const double* part_wa, int64_t n_pwa, const double* part_ws, int64_t n_pws,
+                          const double* ar2_alpha2, const double* ar1_wa, int init, int32_t* host_flag,
+                          cudaStream_t s) {
+  k_scalar<<<1, kRedThreads, 0, s>>>(st, part_astro, n_pa, part_sh, n_ps, part_wa, n_pwa, part_ws, n_pws,
+                                     ar2_alpha2, ar1_wa, init, host_flag);
+  return cudaGetLastError();
+}
+cudaError_t launch_colupdate(double* v, double* w, double* x, double* var, int64_t n, int64_t A0, double* part_wa,
+                             double* part_ws, int nblk, const DevState* st, cudaStream_t s) {
+  k_colupdate<<<nblk, kRedThreads, 0, s>>>(v, w, x, var, n, A0, part_wa, part_ws, st);
+  return cudaGetLastError();
+}
+cudaError_t launch_sum_to(const double* part, int64_t n, double* dst, cudaStream_t s) {
+  k_sum_to<<<1, kRedThreads, 0, s>>>(part, n, dst);
+  return cudaGetLastError();
+}
+cudaError_t launch_precond_D(double* c, int64_t n, cudaStream_t s) {
+  k_precond_D<<<vec_grid(n, 148 * 4), kRedThreads, 0, s>>>(c, n);
+  return cudaGetLastError();
+}
+cudaError_t launch_finalize(const double* x, const double* var, const double* D, int64_t n, const DevState* st,
+                            double se_t, double* x_out, double* se_out, cudaStream_t s) {
+  k_finalize<<<vec_grid(n, 148 * 4), kRedThreads, 0, s>>>(x, var, D, n, st, se_t, x_out, se_out);
+  return cudaGetLastError();
+}
+cudaError_t launch_fill(double* p, int64_t n, double v, cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  k_fill<<<vec_grid(n, 148 * 4), kRedThreads, 0, s>>>(p, n, v);
+  return cudaGetLastError();
+}
+
+}  // namespace lsqr

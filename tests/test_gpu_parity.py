@@ -1,0 +1,310 @@
+"""GPU-vs-oracle parity of the CUDA path, called through the C ABI (SURVEY §8(c) parity contract).
+
+  generator arrays, shard layouts ........ bit-exact
+  single aprod1/aprod2 calls ............. |gpu - oracle| <= 1e-13 * (sum |a_ij x_j| + |y_i|) per element
+  preconditioner D ....................... 1e-14 relative per element (column sums of squares reordered)
+  teacher-forced LSQR step ............... u, v, w, x <= 1e-12 relative (norm), alpha/beta 1e-12
+  free-run u, v .......................... <= 1e-12 for k <= k_div (summation order differs; SURVEY EXP-1/2)
+  converged x (fixed count) .............. <= 1e-9 relative;  r1norm 1e-10;  istop equal
+  standard errors ........................ statistical (median relative difference <= 1e-2)
+"""
+import numpy as np
+import pytest
+
+import oracle
+import workloads as W
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def avu(cuda_device):
+    import paper_conf_sc_malenzacsbvba24_b200 as m
+    return m
+
+
+def gpu_solver(avu, w, **kw):
+    return avu.Solver.synthetic(w, **kw)
+
+
+def abs_system(S):
+    A = oracle.System(S.w, generate=False)
+    A.__dict__.update({k: getattr(S, k) for k in ("star_begin", "star_end", "row_begin", "row_end", "n_rows")})
+    A.vals = np.abs(S.vals); A.mA, A.mT, A.iC = S.mA, S.mT, S.iC
+    A.c_val = np.abs(S.c_val); A.c_ptr, A.c_col = S.c_ptr, S.c_col
+    A.n_constr = S.n_constr
+    A.rank = S.rank
+    A._mk_struct()
+    return A
+
+
+def to_local_x(S, xg):
+    """global column vector -> this rank's local layout [astro of own stars | shared]"""
+    return np.concatenate([xg[5 * S.star_begin:5 * S.star_end], xg[S.A0:]])
+
+
+# ------------------------------------------------------------------------------------------------ generator
+GEN_CASES = [W.C1, W.C1C, W.micro(n_glob=0, seed=5), W.micro(seed=13, b_mode=1, noise=0.25),
+             W.C2.replace(n_stars=20_000, n_obs=2_000_000, seed=7)]
+
+
+@pytest.mark.parametrize("w", GEN_CASES, ids=lambda w: w.name + f"-b{w.b_mode}-g{w.n_glob}")
+def test_generator_bit_exact(avu, w):
+    s = gpu_solver(avu, w)
+    S = oracle.System(w)
+    g = s.get_system()
+    for k in ("vals", "mA", "mT", "iC", "b"):
+        a, b = g[k], getattr(S, k)
+        assert a.shape == b.shape
+        assert np.array_equal(a.view(np.uint8), b.view(np.uint8)), k
+    s.close()
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_sharded_generation_bit_exact(avu, P):
+    w = W.C1C.replace(jitter_pct=50)
+    for r in range(P):
+        s = gpu_solver(avu, w, rank=r, nranks=P, comm="callback", allreduce=lambda *a: 1)
+        S = oracle.System(w, rank=r, nranks=P)
+        assert (s.star_begin, s.star_end, s.row_begin, s.row_end) == (S.star_begin, S.star_end, S.row_begin,
+                                                                       S.row_end)
+        g = s.get_system()
+        for k in ("vals", "mA", "mT", "iC", "b"):
+            assert np.array_equal(g[k], getattr(S, k)), (r, k)
+        s.close()
+
+
+# ------------------------------------------------------------------------------------------------ products
+APROD_CASES = [W.C1, W.C1C, W.micro(n_glob=0, seed=5, n_ext=3), W.micro(n_stars=3, obs=1, jitter=0),
+               W.C2.replace(n_stars=20_000, n_obs=2_000_000, seed=7), W.C1.replace(n_instr=24_000, n_obs=30_000)]
+
+
+def _check(got, ref, scale, tol=1e-13):
+    err = np.abs(got - ref)
+    bad = err > tol * scale
+    assert not bad.any(), f"{bad.sum()} elements off; worst {np.max(err / np.maximum(scale, 1e-300)):.3e}"
+
+
+@pytest.mark.parametrize("precond", [False, True])
+@pytest.mark.parametrize("w", APROD_CASES, ids=lambda w: f"{w.name}-{w.n_obs}-i{w.n_instr}-c{w.n_constr}")
+def test_aprod_parity(avu, w, precond):
+    import torch
+    s = gpu_solver(avu, w)
+    S = oracle.System(w)
+    if precond:
+        s.precondition()
+        S.apply_precond()
+        Dg = s.get_precond()
+        assert np.allclose(Dg, S.D, rtol=1e-14, atol=0)
+        # run the oracle products on the GPU's scaled matrix so both sides see identical inputs
+        g = s.get_system(with_b=False)
+        S.vals[:] = g["vals"]
+        S.c_val[:] = S.c_val  # constraint values: scaled by the oracle's D (differs by rounding only)
+    A = abs_system(S)
+    rng = np.random.default_rng(1)
+    x = rng.standard_normal(S.n_cols)
+    y0 = rng.standard_normal(S.m_local)
+    # aprod1
+    yg = torch.tensor(y0, device="cuda")
+    s.aprod1(torch.tensor(x, device="cuda"), yg)
+    yr = y0.copy(); S.aprod1(x, yr)
+    sc = np.abs(y0); A.aprod1(np.abs(x), sc)
+    _check(yg.cpu().numpy(), yr, sc, 1e-13 if not precond else 1e-12)
+    # aprod2
+    yy = rng.standard_normal(S.m_local)
+    x0 = rng.standard_normal(S.n_cols)
+    xg = torch.tensor(x0, device="cuda")
+    s.aprod2(torch.tensor(yy, device="cuda"), xg)
+    xr = x0.copy(); S.aprod2(yy, xr)
+    sc2 = np.abs(x0); A.aprod2(np.abs(yy), sc2)
+    _check(xg.cpu().numpy(), xr, sc2, 1e-13 if not precond else 1e-12)
+    s.close()
+
+
+def test_aprod_full_C2_parity(avu):
+    """BASELINE configs[1] (C2, 5 M rows, constraints) at full size, launch configuration of the bench."""
+    import torch
+    w = W.C2
+    s = gpu_solver(avu, w)
+    S = oracle.System(w)
+    A = abs_system(S)
+    rng = np.random.default_rng(2)
+    x = rng.standard_normal(S.n_cols)
+    y = np.zeros(S.m_local)
+    yg = torch.zeros(S.m_local, dtype=torch.float64, device="cuda")
+    s.aprod1(torch.tensor(x, device="cuda"), yg)
+    S.aprod1(x, y)
+    sc = np.zeros(S.m_local); A.aprod1(np.abs(x), sc)
+    _check(yg.cpu().numpy(), y, sc)
+    yy = rng.standard_normal(S.m_local)
+    xg = torch.zeros(S.n_cols, dtype=torch.float64, device="cuda")
+    s.aprod2(torch.tensor(yy, device="cuda"), xg)
+    xr = np.zeros(S.n_cols); S.aprod2(yy, xr)
+    sc2 = np.zeros(S.n_cols); A.aprod2(np.abs(yy), sc2)
+    _check(xg.cpu().numpy(), xr, sc2)
+    s.close()
+
+
+# ------------------------------------------------------------------------------------------------ LSQR
+def oracle_trace(S, itn, **kw):
+    hist = []
+    res = oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), itn_limit=itn, fixed_count=True,
+                      trace=lambda st, u, v, w_, x, var: hist.append((st, u, v, w_, x, var)), **kw)
+    return res, hist
+
+
+def rel(a, b):
+    return np.linalg.norm(a - b) / max(np.linalg.norm(b), 1e-300)
+
+
+def reversed_control(S):
+    """Control run of SURVEY §8(c): the same system with every sum in a different order (rows reversed, constraint
+    entries reversed within their row).  Returns the oracle System of the permuted problem."""
+    import copy
+    C2 = copy.copy(S)
+    C2.vals = S.vals[::-1].copy(); C2.mA = S.mA[::-1].copy(); C2.mT = S.mT[::-1].copy(); C2.iC = S.iC[::-1].copy()
+    C2.b = S.b[::-1].copy()
+    cc, cv = S.c_col.copy(), S.c_val.copy()
+    for k in range(S.n_constr):
+        a, b = S.c_ptr[k], S.c_ptr[k + 1]
+        cc[a:b] = S.c_col[a:b][::-1]; cv[a:b] = S.c_val[a:b][::-1]
+    C2.c_col, C2.c_val = cc, cv
+    C2._mk_struct()
+    return C2
+
+
+def free_run_curves(avu, w, kmax=30):
+    s = gpu_solver(avu, w)
+    s.precondition()
+    S = oracle.System(w)
+    S.apply_precond()
+    S.vals[:] = s.get_system(with_b=False)["vals"]   # both sides on the GPU's scaled matrix (identical inputs)
+    res_o, hist = oracle_trace(S, 100, atol=0, btol=0, conlim=0)
+    Cs = reversed_control(S)
+    _, hc = oracle_trace(Cs, kmax, atol=0, btol=0, conlim=0)
+    n = S.n_rows
+    ctrl, gpu = [], []
+    s.init(itn_limit=100, atol=0, btol=0, conlim=0, fixed_count=True)
+    for k in range(1, kmax + 1):
+        s.iterate(1)
+        st, vec = s.get_state()
+        so, u, v, w_, x, var = hist[k - 1]
+        uc = np.concatenate([hc[k - 1][1][:n][::-1], hc[k - 1][1][n:]])
+        ctrl.append(max(rel(uc, u), rel(hc[k - 1][2], v)))
+        gpu.append(max(rel(vec["u"], u), rel(vec["v"], v)))
+        assert st["itn"] == k
+    return s, S, res_o, np.array(ctrl), np.array(gpu)
+
+
+@pytest.mark.parametrize("w", [W.C1, W.C1C], ids=["C1", "C1c"])
+def test_lsqr_free_run_and_converged(avu, w):
+    s, S, res_o, ctrl, gpu = free_run_curves(avu, w)
+    print("\nfree-run rel diff per iteration (control = oracle with reordered sums | GPU):")
+    for k, (c, g) in enumerate(zip(ctrl, gpu), 1):
+        print(f"  k={k:2d}  control {c:.2e}  gpu {g:.2e}")
+    k_div = int(np.argmax(ctrl > 1e-12)) + 1 if (ctrl > 1e-12).any() else len(ctrl) + 1
+    # u, v agree to 1e-12 well before the intrinsic divergence onset, and grow no faster than the control
+    k_ok = max(3, k_div - 6)
+    assert (gpu[:k_ok] <= 1e-12).all(), (k_div, gpu[:k_ok])
+    assert (gpu[:k_div - 1] <= 1e3 * np.maximum(ctrl[:k_div - 1], 1e-15)).all()
+    s.iterate(100 - len(gpu))
+    out = s.finalize()
+    assert out["itn"] == 100
+    xo = S.D * res_o["x"]
+    assert rel(out["x"], xo) <= 1e-9
+    assert abs(out["r1norm"] - res_o["r1norm"]) <= 1e-10 * res_o["r1norm"]
+    assert abs(out["arnorm"] - res_o["arnorm"]) <= 1e-10 * res_o["anorm"] * res_o["r1norm"]
+    assert out["istop_first"] == res_o["istop_first"]
+    seo = S.D * res_o["se"]
+    d = np.abs(out["se"] / seo - 1)
+    assert np.median(d) <= 1e-2
+    s.close()
+
+
+@pytest.mark.parametrize("w", [W.C1, W.C1C], ids=["C1", "C1c"])
+def test_lsqr_teacher_forced_step(avu, w):
+    s = gpu_solver(avu, w)
+    s.precondition()
+    S = oracle.System(w)
+    S.apply_precond()
+    S.vals[:] = s.get_system(with_b=False)["vals"]
+    _, hist = oracle_trace(S, 60, atol=0, btol=0, conlim=0)
+    s.init(itn_limit=1000, atol=0, btol=0, conlim=0, fixed_count=True)
+    for k in (1, 2, 5, 13, 30, 59):
+        so, u, v, w_, x, var = hist[k - 1]
+        sc = dict(so); sc["itn"] = k; sc["istop"] = 0; sc["istop_first"] = 0; sc["halted"] = 0
+        s.set_state(sc, u=u, v=v, w=w_, x=x, var=var)
+        s.iterate(1)
+        st, vec = s.get_state()
+        sn, un, vn, wn, xn, varn = hist[k]
+        assert st["itn"] == k + 1
+        for a, b, name in ((vec["u"], un, "u"), (vec["v"], vn, "v"), (vec["w"], wn, "w"), (vec["x"], xn, "x")):
+            assert rel(a, b) <= 1e-12, (k, name, rel(a, b))
+        for name in ("alpha", "beta", "phibar", "rhobar"):
+            assert abs(st[name] - sn[name]) <= 1e-12 * abs(sn[name]) + 1e-300, (k, name)
+    s.close()
+
+
+def test_lsqr_solve_api_and_stopping(avu):
+    w = W.C1
+    s = gpu_solver(avu, w)
+    s.precondition()
+    S = oracle.System(w)
+    S.apply_precond()
+    S.vals[:] = s.get_system(with_b=False)["vals"]
+    ro = oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), atol=1e-10, btol=1e-10, itn_limit=500)
+    out = s.solve(itn_limit=500, atol=1e-10, btol=1e-10)
+    assert out["istop"] == ro["istop"] and abs(out["itn"] - ro["itn"]) <= 2
+    assert rel(out["x"], S.D * ro["x"]) <= 1e-8
+    # b was consumed
+    with pytest.raises(avu.LsqrError):
+        s.solve(itn_limit=5)
+    # a regenerated system (preconditioning reset) reproduces the solve
+    s.generate(w.seed)
+    s.precondition()
+    out2 = s.solve(itn_limit=500, atol=1e-10, btol=1e-10)
+    assert out2["itn"] == out["itn"] and rel(out2["x"], out["x"]) <= 1e-12
+    s.close()
+
+
+def test_lsqr_special_cases(avu):
+    w = W.micro(n_stars=40, obs=30, seed=4)
+    s = gpu_solver(avu, w)
+    S = oracle.System(w)
+    g = s.get_system()
+    s.set_system(g["vals"], g["mA"], g["mT"], g["iC"], np.zeros(S.n_rows))
+    out = s.solve(itn_limit=10)
+    assert out["istop"] == 0 and out["itn"] == 0 and not out["x"].any()
+    s.set_system(g["vals"], g["mA"], g["mT"], g["iC"], g["b"])
+    out = s.solve(itn_limit=4, atol=0, btol=0, conlim=0)
+    assert out["istop"] == 7 and out["itn"] == 4
+    s.close()
+    wp = W.micro(n_stars=40, obs=30, seed=13, b_mode=1, noise=0.0)
+    s = gpu_solver(avu, wp)
+    out = s.solve(itn_limit=2000, atol=1e-14, btol=1e-14, conlim=0)
+    assert out["istop"] == 1
+    xt = oracle.x_true(wp)
+    assert rel(out["x"], xt) <= 1e-9
+    s.close()
+
+
+def test_lsqr_damped(avu):
+    w = W.micro(n_stars=30, obs=25, seed=11)
+    s = gpu_solver(avu, w)
+    S = oracle.System(w)
+    ro = oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), damp=0.3, atol=1e-14, btol=1e-14, conlim=0, itn_limit=400)
+    out = s.solve(itn_limit=400, atol=1e-14, btol=1e-14, conlim=0, damp=0.3)
+    assert rel(out["x"], ro["x"]) <= 1e-9
+    assert abs(out["r1norm"] - ro["r1norm"]) <= 1e-9 * ro["r1norm"]
+    s.close()
+
+
+def test_graph_and_eager_agree(avu):
+    w = W.C1C
+    outs = []
+    for g in (True, False):
+        s = gpu_solver(avu, w)
+        s.precondition()
+        outs.append(s.solve(itn_limit=30, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=g))
+        s.close()
+    assert rel(outs[0]["x"], outs[1]["x"]) <= 1e-10

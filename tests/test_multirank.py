@@ -1,0 +1,174 @@
+"""Multi-rank path: rows sharded by star, shared slice + scalar norms allreduced.
+
+CPU (gloo, world_size 2, run here): each process takes its O-SHARD star range from the PRODUCT's host shard map,
+checks it against the oracle bit-exactly, runs the oracle products on its own shard and combines them with a real
+gloo allreduce (AR1: constraint dots; AR2: shared slice), which must equal the single-rank products -- i.e. the
+decomposition the CUDA path implements is exact.
+
+GPU (gloo host-callback communicator, 2 processes sharing cuda:0): the product's multi-rank LSQR (AR1/AR2 through
+the C ABI's allreduce hook) against the single-rank GPU run and the oracle.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch.multiprocessing as mp
+
+import workloads as W
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _init(rank, world, port):
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    return dist
+
+
+def _cpu_worker(rank, world, port, q):
+    try:
+        import sys
+        sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+        import torch
+        import oracle
+        import paper_conf_sc_malenzacsbvba24_b200 as avu
+        dist = _init(rank, world, port)
+        w = W.C1C.replace(n_stars=300, n_obs=6000, jitter_pct=50, n_ext_stars=200, seed=17)
+        counts = avu.synth_obs_per_star(w.seed, w.n_stars, w.n_obs, w.jitter_pct)
+        sb = avu.shard_map(counts, w.n_obs, world)
+        S = oracle.System(w, rank=rank, nranks=world)
+        assert (sb[rank], sb[rank + 1]) == (S.star_begin, S.star_end)
+        rng = np.random.default_rng(5)
+        x = rng.standard_normal(S.n_cols)
+        y_full = rng.standard_normal(w.n_obs + S.n_constr)
+        # aprod1: local rows + owned constraint partial dots, AR1 over the constraint part
+        yl = np.zeros(S.m_local)
+        S.aprod1(x, yl)
+        c = torch.tensor(yl[S.n_rows:])
+        dist.all_reduce(c)
+        # aprod2: local astro + shared partial, AR2 over the shared slice
+        yr = np.concatenate([y_full[S.row_begin:S.row_end], y_full[w.n_obs:]])
+        xl = np.zeros(S.n_cols)
+        S.aprod2(yr, xl)
+        sh = torch.tensor(xl[S.A0:])
+        dist.all_reduce(sh)
+        q.put((rank, S.row_begin, yl[:S.n_rows], c.numpy(), S.star_begin, S.star_end, xl[:S.A0], sh.numpy()))
+        dist.destroy_process_group()
+    except Exception as e:  # pragma: no cover
+        import traceback
+        q.put(("error", traceback.format_exc()))
+
+
+def test_gloo_two_rank_decomposition_cpu():
+    import oracle
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_cpu_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    outs = [q.get(timeout=180) for _ in range(2)]
+    for p in ps:
+        p.join(60)
+    for o in outs:
+        assert o[0] != "error", o[1]
+    w = W.C1C.replace(n_stars=300, n_obs=6000, jitter_pct=50, n_ext_stars=200, seed=17)
+    S = oracle.System(w)
+    rng = np.random.default_rng(5)
+    x = rng.standard_normal(S.n_cols)
+    y_full = rng.standard_normal(w.n_obs + S.n_constr)
+    y1 = np.zeros(S.m_local); S.aprod1(x, y1)
+    x2 = np.zeros(S.n_cols); S.aprod2(y_full, x2)
+    got_y = np.zeros(S.m_local)
+    got_x = np.zeros(S.n_cols)
+    for (rank, rb, yrows, cdots, sb, se, xast, xsh) in outs:
+        got_y[rb:rb + len(yrows)] = yrows
+        got_y[S.n_rows:] = cdots  # identical on both ranks after AR1
+        got_x[5 * sb:5 * se] = xast[5 * sb:5 * se]
+        got_x[S.A0:] = xsh
+    assert np.allclose(got_y, y1, rtol=1e-14, atol=1e-13)
+    assert np.allclose(got_x, x2, rtol=1e-13, atol=1e-13)
+
+
+# ------------------------------------------------------------------------------------------------ GPU
+def _gpu_worker(rank, world, port, q, itn):
+    try:
+        import sys
+        sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+        import torch
+        import paper_conf_sc_malenzacsbvba24_b200 as avu
+        _init(rank, world, port)
+        torch.cuda.set_device(0)
+        w = W.C1C.replace(jitter_pct=50)
+        s = avu.Solver.synthetic(w, rank=rank, nranks=world, comm="callback")
+        s.precondition()
+        D = s.get_precond()
+        out = s.solve(itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=False)
+        # plain products through the ABI
+        xg = torch.ones(s.n_local_cols, dtype=torch.float64, device="cuda")
+        yg = torch.zeros(s.n_local_rows + s.n_constr, dtype=torch.float64, device="cuda")
+        s.aprod1(xg, yg)
+        x2 = torch.zeros_like(xg)
+        s.aprod2(torch.ones_like(yg), x2)
+        q.put((rank, s.star_begin, s.star_end, s.row_begin, out["x"], out["se"], out["itn"], out["r1norm"], D,
+               yg.cpu().numpy(), x2.cpu().numpy()))
+        s.close()
+        import torch.distributed as dist
+        dist.destroy_process_group()
+    except Exception:
+        import traceback
+        q.put(("error", traceback.format_exc()))
+
+
+@pytest.mark.gpu
+def test_gpu_two_rank_lsqr_matches_single_rank(cuda_device):
+    import torch
+    import paper_conf_sc_malenzacsbvba24_b200 as avu
+    itn = 60
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_gpu_worker, args=(r, 2, port, q, itn)) for r in range(2)]
+    for p in ps:
+        p.start()
+    outs = [q.get(timeout=600) for _ in range(2)]
+    for p in ps:
+        p.join(60)
+    for o in outs:
+        assert o[0] != "error", o[1]
+    w = W.C1C.replace(jitter_pct=50)
+    s = avu.Solver.synthetic(w)
+    s.precondition()
+    D1 = s.get_precond()
+    ref = s.solve(itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True)
+    xg = torch.ones(s.n_local_cols, dtype=torch.float64, device="cuda")
+    yg = torch.zeros(s.n_local_rows + s.n_constr, dtype=torch.float64, device="cuda")
+    s.aprod1(xg, yg)
+    x2 = torch.zeros_like(xg)
+    s.aprod2(torch.ones_like(yg), x2)
+    y1, x21 = yg.cpu().numpy(), x2.cpu().numpy()
+    A0 = 5 * w.n_stars
+    n_rows = w.n_obs
+    for (rank, sb, se, rb, x, sev, it, r1, D, y, xx) in outs:
+        A0l = 5 * (se - sb)
+        glob = lambda v: (v[:A0l], v[A0l:])
+        xa, xs = glob(x)
+        assert it == itn
+        assert np.allclose(D[:A0l], D1[5 * sb:5 * se], rtol=1e-14) and np.allclose(D[A0l:], D1[A0:], rtol=1e-14)
+        rel = lambda a, b: np.linalg.norm(a - b) / np.linalg.norm(b)
+        assert rel(xa, ref["x"][5 * sb:5 * se]) <= 1e-9 and rel(xs, ref["x"][A0:]) <= 1e-9
+        assert abs(r1 - ref["r1norm"]) <= 1e-10 * ref["r1norm"]
+        assert np.allclose(y[:len(y) - 12], y1[rb:rb + len(y) - 12], rtol=1e-12, atol=1e-12)
+        assert np.allclose(y[-12:], y1[n_rows:], rtol=1e-12, atol=1e-12)
+        assert np.allclose(xx[:A0l], x21[5 * sb:5 * se], rtol=1e-12, atol=1e-12)
+        assert np.allclose(xx[A0l:], x21[A0:], rtol=1e-12, atol=1e-12)
+    s.close()
