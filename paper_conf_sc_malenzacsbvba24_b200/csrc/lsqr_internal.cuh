@@ -7,10 +7,16 @@
 namespace lsqr {
 
 constexpr int kSlots = 24;           // 5 astro + 12 att + 6 instr + 1 glob
-constexpr int kThreads = 768;        // persistent row kernels: one 24-warp CTA per SM (80 regs/thread)
+
+constexpr int kThreads = 384;        // persistent row kernels: one 12-warp CTA per SM
 constexpr int kWarpsPerCta = kThreads / 32;
+constexpr int kRows = 16;            // rows per TMA stage (two 8-row groups, 4 lanes per row)
+constexpr int kStages = 4;           // ring depth per warp (kStages-1 stages in flight while computing)
+constexpr int kStageBytes = kRows * (kSlots * 8 + 16);                  // 3328 B: values + index records
+constexpr int kRingBytes = kWarpsPerCta * kStages * kStageBytes;        // 159,744 B per CTA
+constexpr int kBarBytes = kWarpsPerCta * kStages * 8;                   // mbarriers
 constexpr int kRedThreads = 256;     // small reduction / vector kernels
-constexpr int kInstrSmemMax = 16384; // n_instr above this -> instrumental scatter goes to L2 REDs (no smem)
+constexpr int kInstrSmemMax = 8192;  // n_instr above this -> instrumental scatter goes to L2 REDs (no smem)
 constexpr int kMaxConstr = 64;       // constraint rows handled by the one-block beta kernel
 
 // Per-row index record, 16 B: the paper's matrixIndexAtt (as k0, relative to the attitude block) and instrCol

