@@ -689,9 +689,21 @@ int lsqr_set_system(lsqr_t h, const double* vals, const int64_t* mA, const int64
       rec[i].ic45 = ic[4] | (ic[5] << 16);
     }
   }
+  // paper slot order -> lane-major device order (position 6j + t holds slot_of(t, j)), in row blocks
   enter(h);
   CKR(reset_precond(h));
-  CKC(h, cudaMemcpyAsync(h->vals, vals, sizeof(double) * kSlots * n, cudaMemcpyHostToDevice, h->s));
+  {
+    const int64_t blk = 1 << 16;
+    std::vector<double> tmp(std::max<int64_t>(std::min(n, blk), 1) * kSlots);
+    for (int64_t r0 = 0; r0 < n; r0 += blk) {
+      const int64_t nb = std::min(blk, n - r0);
+      for (int64_t i = 0; i < nb; ++i)
+        for (int p = 0; p < kSlots; ++p) tmp[i * kSlots + p] = vals[(r0 + i) * kSlots + slot_of(p % 6, p / 6)];
+      CKC(h, cudaMemcpyAsync(h->vals + r0 * kSlots, tmp.data(), sizeof(double) * kSlots * nb,
+                             cudaMemcpyHostToDevice, h->s));
+      CKC(h, cudaStreamSynchronize(h->s));
+    }
+  }
   CKC(h, cudaMemcpyAsync(h->idx, rec.data(), sizeof(IdxRec) * n, cudaMemcpyHostToDevice, h->s));
   CKC(h, cudaMemcpyAsync(h->u, b, sizeof(double) * n, cudaMemcpyHostToDevice, h->s));
   CKC(h, cudaStreamSynchronize(h->s));  // rec is a temporary
@@ -709,7 +721,14 @@ int lsqr_get_system(lsqr_t h, double* vals, int64_t* mA, int64_t* mT, int64_t* i
   const int64_t n = h->n_loc_rows;
   enter(h);
   CKC(h, cudaStreamSynchronize(h->s));
-  if (vals) CKC(h, cudaMemcpy(vals, h->vals, sizeof(double) * kSlots * n, cudaMemcpyDeviceToHost));
+  if (vals) {
+    CKC(h, cudaMemcpy(vals, h->vals, sizeof(double) * kSlots * n, cudaMemcpyDeviceToHost));
+    double row[kSlots];
+    for (int64_t i = 0; i < n; ++i) {  // lane-major -> paper slot order
+      for (int p = 0; p < kSlots; ++p) row[slot_of(p % 6, p / 6)] = vals[i * kSlots + p];
+      memcpy(vals + i * kSlots, row, sizeof row);
+    }
+  }
   if (b) CKC(h, cudaMemcpy(b, h->u, sizeof(double) * n, cudaMemcpyDeviceToHost));
   if (mA || mT || iC) {
     std::vector<IdxRec> rec(std::max<int64_t>(n, 1));

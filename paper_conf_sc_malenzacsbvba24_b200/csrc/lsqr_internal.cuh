@@ -8,9 +8,10 @@ namespace lsqr {
 
 constexpr int kSlots = 24;           // 5 astro + 12 att + 6 instr + 1 glob
 
-constexpr int kThreads = 384;        // persistent row kernels: one 12-warp CTA per SM
+constexpr int kThreads = 768;        // persistent row kernels: one 24-warp CTA per SM
 constexpr int kWarpsPerCta = kThreads / 32;
-constexpr int kRows = 16;            // rows per TMA stage (two 8-row groups, 4 lanes per row)
+constexpr int kRows = 8;             // rows per TMA stage (one 8-row group, 4 lanes per row)
+constexpr int kGroups = kRows / 8;
 constexpr int kStages = 4;           // ring depth per warp (kStages-1 stages in flight while computing)
 constexpr int kStageBytes = kRows * (kSlots * 8 + 16);                  // 3328 B: values + index records
 constexpr int kRingBytes = kWarpsPerCta * kStages * kStageBytes;        // 159,744 B per CTA
@@ -18,6 +19,14 @@ constexpr int kBarBytes = kWarpsPerCta * kStages * 8;                   // mbarr
 constexpr int kRedThreads = 256;     // small reduction / vector kernels
 constexpr int kInstrSmemMax = 8192;  // n_instr above this -> instrumental scatter goes to L2 REDs (no smem)
 constexpr int kMaxConstr = 64;       // constraint rows handled by the one-block beta kernel
+constexpr int kMaxChunksSmem = 1024; // constraint chunk partials staged in shared memory by k_beta
+
+// Row storage is LANE-MAJOR: the 24 values of a row are stored so that lane j of the row's 4-lane group finds its
+// 6 values at positions 6j..6j+5 (slot_of(t, j) = slot held at position 6j + t).  Slot 23 stays at position 23.
+// lsqr_set_system / lsqr_get_system convert from / to the paper's slot order.
+__host__ __device__ __forceinline__ int slot_of(int t, int j) {
+  return t == 0 ? j : (t <= 3 ? 5 + 4 * (t - 1) + j : (t == 4 ? 17 + j : (j == 0 ? 4 : 20 + j)));
+}
 
 // Per-row index record, 16 B: the paper's matrixIndexAtt (as k0, relative to the attitude block) and instrCol
 // (6 x u16, relative to the instrumental block) in one 128-bit word.  matrixIndexAstro is implicit: rows are

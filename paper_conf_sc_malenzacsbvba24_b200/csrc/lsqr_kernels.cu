@@ -46,10 +46,6 @@ __device__ __forceinline__ uint32_t ic_of(const IdxRec& r, int q) {  // instrCol
   return (w >> ((q & 1) * 16)) & 0xffffu;
 }
 
-__device__ __forceinline__ int slot_of(int t, int j) {
-  return t == 0 ? j : (t <= 3 ? 5 + 4 * (t - 1) + j : (t == 4 ? 17 + j : (j == 0 ? 4 : 20 + j)));
-}
-
 // ------------------------------------------------------------------------------------------------ generator
 // O-GEN (docs/GENERATOR.md): splitmix64-based counter hash; integer-only, exact int->double conversions, so the
 // device arrays are bit-identical to any other implementation of the spec.
@@ -95,9 +91,10 @@ __global__ void k_generate(GenArgs g, double* __restrict__ vals, IdxRec* __restr
 #pragma unroll
     for (int s = 0; s < kSlots; ++s) v[s] = g_pm1(g_hash(g.seed, 4, i, s));
     if (g.n_glob == 0) v[23] = 0.0;
-    double* rp = vals + li * kSlots;
+    double* rp = vals + li * kSlots;  // lane-major storage (position 6j + t holds slot_of(t, j))
 #pragma unroll
-    for (int s = 0; s < kSlots; s += 2) *reinterpret_cast<double2*>(rp + s) = make_double2(v[s], v[s + 1]);
+    for (int p = 0; p < kSlots; p += 2)
+      *reinterpret_cast<double2*>(rp + p) = make_double2(v[slot_of(p % 6, p / 6)], v[slot_of((p + 1) % 6, p / 6)]);
     if (g.b_mode == 0) {
       b[li] = g_pm1(g_hash(g.seed, 5, i, 0));
     } else {  // planted: b = sum_s val_s * x_true[col_s] in slot order, every op rounded (no FMA), + noise term
@@ -203,9 +200,14 @@ __device__ __forceinline__ const unsigned char* ring_wait(const Ring& R, int64_t
 
 // row lr (0..kRows-1) of a stage: the lane's 6 values and the index record (16-B broadcast within the row group)
 __device__ __forceinline__ void stage_row(const unsigned char* stg, int lr, int j, double (&v)[6], IdxRec& rec) {
-  const double* rp = reinterpret_cast<const double*>(stg + lr * kSlots * 8);
+  // lane-major row: the lane's 6 values are 48 contiguous bytes -> three conflict-free 16-B shared loads
+  const double2* rp = reinterpret_cast<const double2*>(stg + lr * kSlots * 8 + 48 * j);
 #pragma unroll
-  for (int t = 0; t < 6; ++t) v[t] = rp[slot_of(t, j)];
+  for (int q = 0; q < 3; ++q) {
+    const double2 d = rp[q];
+    v[2 * q] = d.x;
+    v[2 * q + 1] = d.y;
+  }
   const int4 q = *reinterpret_cast<const int4*>(stg + kRows * kSlots * 8 + lr * 16);
   rec.k0 = q.x;
   rec.ic01 = (uint32_t)q.y; rec.ic23 = (uint32_t)q.z; rec.ic45 = (uint32_t)q.w;
@@ -231,12 +233,18 @@ __device__ __forceinline__ void track_star(const SysView& S, int64_t row, int64_
 // MODE AP1_LSQR:  u_hat[i] = sum_s a_is v[col_is] - u_scale * u_hat[i];  per-warp partial of u_hat^2 (beta^2).
 // MODE AP1_PLAIN: y[i] += sum_s a_is x[col_is].
 // Constraint rows: per-chunk partial dots of the owned entries -> cpart (combined by k_beta / k_cdot).
-template <int MODE>
+template <int MODE, bool SMEM_INSTR>
 __global__ void __launch_bounds__(kThreads, 1)
     k_aprod1(SysView S, const double* __restrict__ x, double* __restrict__ y, double* __restrict__ part,
              double* __restrict__ cpart, const DevState* __restrict__ st) {
   extern __shared__ __align__(128) unsigned char dsm[];
   if (MODE == AP1_LSQR && st->halted) return;
+  // the instrumental slice of x (<= 64 KB) is staged in shared memory: its gathers are random and L1-hostile
+  double* sh_x = reinterpret_cast<double*>(dsm + kRingBytes + kBarBytes);
+  if (SMEM_INSTR) {
+    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_x[i] = x[S.I0 + i];
+    __syncthreads();
+  }
   const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2, wid = threadIdx.x >> 5;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -247,25 +255,26 @@ __global__ void __launch_bounds__(kThreads, 1)
   const bool glob_ok = S.n_glob != 0;
   int64_t s = s_lo, bound = S.star_ptr[s_lo + 1];
   double b2 = 0.0;
-  double ynext[2];
+  double ynext[kGroups];
 #pragma unroll
-  for (int q = 0; q < 2; ++q) {
+  for (int q = 0; q < kGroups; ++q) {
     const int64_t row = R.r_lo + q * 8 + r;
     ynext[q] = row < R.r_hi ? __ldg(y + row) : 0.0;
   }
   for (int64_t k = 0; k < R.nst; ++k) {
     const int64_t row0 = R.r_lo + k * kRows;
-    double ycur[2] = {ynext[0], ynext[1]};
+    double ycur[kGroups];
 #pragma unroll
-    for (int q = 0; q < 2; ++q) {  // prefetch next stage's y (u_hat)
+    for (int q = 0; q < kGroups; ++q) {  // prefetch next stage's y (u_hat)
+      ycur[q] = ynext[q];
       const int64_t row = row0 + kRows + q * 8 + r;
       ynext[q] = row < R.r_hi ? __ldg(y + row) : 0.0;
     }
     const unsigned char* stg = ring_wait(R, k);
-    double v[2][6], xv[2][6];
-    bool valid[2];
+    double v[kGroups][6], xv[kGroups][6];
+    bool valid[kGroups];
 #pragma unroll
-    for (int q = 0; q < 2; ++q) {
+    for (int q = 0; q < kGroups; ++q) {
       const int64_t row = row0 + q * 8 + r;
       valid[q] = row < R.r_hi;
       IdxRec rec;
@@ -274,12 +283,14 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
       for (int t = 0; t < 6; ++t) {
         const bool ok = valid[q] && !(t == 5 && j == 3 && !glob_ok);
-        xv[q][t] = ok ? __ldg(x + col_of(S, t, j, s, rec)) : 0.0;
+        const bool in_smem = SMEM_INSTR && (t == 4 || (t == 5 && (j == 1 || j == 2)));
+        if (in_smem) xv[q][t] = ok ? sh_x[ic_of(rec, t == 4 ? j : 3 + j)] : 0.0;
+        else xv[q][t] = ok ? __ldg(x + col_of(S, t, j, s, rec)) : 0.0;
       }
     }
     ring_release(S, R, k, lane);
 #pragma unroll
-    for (int q = 0; q < 2; ++q) {
+    for (int q = 0; q < kGroups; ++q) {
       double p = 0.0;
 #pragma unroll
       for (int t = 0; t < 6; ++t) p = fma(v[q][t], xv[q][t], p);
@@ -386,23 +397,24 @@ __global__ void __launch_bounds__(kThreads, 1)
   };
 
   const double* ysrc = MODE == AP2_COLNORM ? nullptr : yv;
-  double ynext[2];
+  double ynext[kGroups];
 #pragma unroll
-  for (int q = 0; q < 2; ++q) {
+  for (int q = 0; q < kGroups; ++q) {
     const int64_t row = R.r_lo + q * 8 + r;
     ynext[q] = (ysrc && row < R.r_hi) ? __ldg(ysrc + row) : 0.0;
   }
   for (int64_t k = 0; k < R.nst; ++k) {
     const int64_t row0 = R.r_lo + k * kRows;
-    double ycur[2] = {ynext[0], ynext[1]};
+    double ycur[kGroups];
 #pragma unroll
-    for (int q = 0; q < 2; ++q) {
+    for (int q = 0; q < kGroups; ++q) {
+      ycur[q] = ynext[q];
       const int64_t row = row0 + kRows + q * 8 + r;
       ynext[q] = (ysrc && row < R.r_hi) ? __ldg(ysrc + row) : 0.0;
     }
     const unsigned char* stg = ring_wait(R, k);
 #pragma unroll
-    for (int q = 0; q < 2; ++q) {
+    for (int q = 0; q < kGroups; ++q) {
       const int64_t base = row0 + q * 8;
       const int64_t row = base + r;
       const bool valid = row < R.r_hi;
@@ -487,12 +499,11 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (row >= r_hi) continue;
     while (S.star_ptr[s + 1] <= row) ++s;
     const IdxRec rec = S.idx[row];
-    double* rp = vals + row * kSlots;
+    double* rp = vals + row * kSlots + 6 * j;  // lane-major: position 6j + t
 #pragma unroll
     for (int t = 0; t < 6; ++t) {
       if (t == 5 && j == 3 && S.n_glob == 0) continue;
-      const int sl = slot_of(t, j);
-      rp[sl] = rp[sl] * D[col_of(S, t, j, s, rec)];
+      rp[t] = rp[t] * D[col_of(S, t, j, s, rec)];
     }
   }
 }
@@ -518,7 +529,7 @@ __global__ void __launch_bounds__(kRedThreads)
     k_beta(int phase, SysView S, const double* __restrict__ part, int64_t n_part, const double* __restrict__ cpart,
            double* __restrict__ ar1, double* __restrict__ uc, double* __restrict__ ucn,
            const double* __restrict__ crhs, DevState* __restrict__ st, int init) {
-  __shared__ double cdot_sh[64];
+  __shared__ double cdot_sh[kMaxConstr];
   __shared__ double b2_sh;
   if (phase != 3 && !init && st->halted) return;
   const int nc = S.n_constr;
@@ -526,11 +537,22 @@ __global__ void __launch_bounds__(kRedThreads)
     const double b2 = phase == 3 ? 0.0 : ordered_sum<kRedThreads>(part, n_part);
     if (threadIdx.x == 0) b2_sh = b2;
     // chunk partials -> per-row dots (chunks are in row order; each row's chunks summed in order)
+    __shared__ double cp_sh[kMaxChunksSmem];
+    __shared__ int32_t cr_sh[kMaxChunksSmem];
+    const int64_t nch = init ? 0 : S.n_chunks;
+    const bool in_smem = nch <= kMaxChunksSmem;
+    if (in_smem)
+      for (int64_t c = threadIdx.x; c < nch; c += blockDim.x) {
+        cp_sh[c] = cpart[c];
+        cr_sh[c] = S.ch_row[c];
+      }
+    __syncthreads();
     if (threadIdx.x < nc) {
       double d = 0.0;
-      if (!init)
-        for (int64_t c = 0; c < S.n_chunks; ++c)
-          if (S.ch_row[c] == (int)threadIdx.x) d += cpart[c];
+      for (int64_t c = 0; c < nch; ++c) {
+        const int rw = in_smem ? cr_sh[c] : S.ch_row[c];
+        if (rw == (int)threadIdx.x) d += in_smem ? cp_sh[c] : cpart[c];
+      }
       cdot_sh[threadIdx.x] = d;
     }
     __syncthreads();
@@ -544,12 +566,15 @@ __global__ void __launch_bounds__(kRedThreads)
     if (threadIdx.x == 0) b2_sh = ar1[nc];
     __syncthreads();
   }
+  __shared__ double uc_sh[kMaxConstr];
+  if (threadIdx.x < nc) uc_sh[threadIdx.x] = init ? (crhs ? crhs[threadIdx.x] : 0.0) : uc[threadIdx.x];
+  __syncthreads();
   if (threadIdx.x == 0) {
     const double us = st->u_scale;
     double b2 = b2_sh;
     for (int k = 0; k < nc; ++k) {
-      const double un = init ? (crhs ? crhs[k] : 0.0) : cdot_sh[k] - us * uc[k];
-      uc[k] = un;
+      const double un = init ? uc_sh[k] : cdot_sh[k] - us * uc_sh[k];
+      uc_sh[k] = un;
       b2 = fma(un, un, b2);
     }
     const double beta = sqrt(b2);
@@ -564,7 +589,12 @@ __global__ void __launch_bounds__(kRedThreads)
     st->beta = beta;
     st->beta_pos = pos;
     st->inv_beta = ib;
-    for (int k = 0; k < nc; ++k) ucn[k] = uc[k] * ib;
+  }
+  __syncthreads();
+  if (threadIdx.x < nc) {
+    const double ib = st->inv_beta;
+    uc[threadIdx.x] = uc_sh[threadIdx.x];
+    ucn[threadIdx.x] = uc_sh[threadIdx.x] * ib;
   }
 }
 
@@ -631,6 +661,9 @@ __global__ void __launch_bounds__(kRedThreads)
   if (threadIdx.x != 0) return;
   if (bp && ar2_alpha2) a2 += *ar2_alpha2;
   if (!init && ar1_wa) w2 += *ar1_wa;
+  DevState* const gst = st;
+  DevState L = *gst;  // all loads issued together; computed on registers, written back once
+  st = &L;
   const double eps = 0x1p-52;
   if (init) {
     const double alpha = bp ? sqrt(a2) : 0.0;
@@ -723,7 +756,8 @@ __global__ void __launch_bounds__(kRedThreads)
     st->u_scale = alpha * st->inv_beta;
     if ((is != 0 && !st->fixed_count) || st->itn >= st->itn_limit) st->halted = 1;
   }
-  if (host_flag) *reinterpret_cast<volatile int32_t*>(host_flag) = st->halted | (st->itn << 1);
+  *gst = L;
+  if (host_flag) *reinterpret_cast<volatile int32_t*>(host_flag) = L.halted | (L.itn << 1);
 }
 
 // O-3e: v <- v/alpha (if pending); d = t3 w; var += d^2; x += t1 w; w = v + t2 w;  partials of ||w_new||^2 split
@@ -795,20 +829,28 @@ cudaError_t launch_generate(const GenArgs& g, double* vals, IdxRec* idx, const i
   return cudaGetLastError();
 }
 
+template <int MODE, bool SM>
+static cudaError_t ap1(const SysView& S, int grid, const double* x, double* y, double* part, double* cpart,
+                       const DevState* st, cudaStream_t s) {
+  const size_t smem = kRingBytes + kBarBytes + (SM ? (size_t)S.n_instr * sizeof(double) : 0);
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(k_aprod1<MODE, SM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)(kRingBytes + kBarBytes + (SM ? kInstrSmemMax * sizeof(double) : 0)));
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  k_aprod1<MODE, SM><<<grid, kThreads, smem, s>>>(S, x, y, part, cpart, st);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_aprod1(int mode, const SysView& S, int grid, const double* x, double* y, double* part,
                           double* cpart, const DevState* st, cudaStream_t s) {
-  static bool attr = false;
-  if (!attr) {
-    for (auto fn : {k_aprod1<AP1_LSQR>, k_aprod1<AP1_PLAIN>}) {
-      cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, kRingBytes + kBarBytes);
-      if (e != cudaSuccess) return e;
-    }
-    attr = true;
-  }
-  const size_t smem = kRingBytes + kBarBytes;
-  if (mode == AP1_LSQR) k_aprod1<AP1_LSQR><<<grid, kThreads, smem, s>>>(S, x, y, part, cpart, st);
-  else k_aprod1<AP1_PLAIN><<<grid, kThreads, smem, s>>>(S, x, y, part, cpart, st);
-  return cudaGetLastError();
+  const bool sm = S.n_instr <= kInstrSmemMax;
+  if (mode == AP1_LSQR) return sm ? ap1<AP1_LSQR, true>(S, grid, x, y, part, cpart, st, s)
+                                  : ap1<AP1_LSQR, false>(S, grid, x, y, part, cpart, st, s);
+  return sm ? ap1<AP1_PLAIN, true>(S, grid, x, y, part, cpart, st, s)
+            : ap1<AP1_PLAIN, false>(S, grid, x, y, part, cpart, st, s);
 }
 
 template <int MODE, bool SM>
