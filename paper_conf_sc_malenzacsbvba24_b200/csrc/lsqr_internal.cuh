@@ -8,11 +8,11 @@ namespace lsqr {
 
 constexpr int kSlots = 24;           // 5 astro + 12 att + 6 instr + 1 glob
 
-constexpr int kThreads = 768;        // persistent row kernels: one 24-warp CTA per SM
+constexpr int kThreads = 512;        // persistent row kernels: one 16-warp CTA per SM
 constexpr int kWarpsPerCta = kThreads / 32;
-constexpr int kRows = 8;             // rows per TMA stage (one 8-row group, 4 lanes per row)
+constexpr int kRows = 16;            // rows per TMA stage (two 8-row groups, 4 lanes per row)
 constexpr int kGroups = kRows / 8;
-constexpr int kStages = 4;           // ring depth per warp (kStages-1 stages in flight while computing)
+constexpr int kStages = 3;           // ring depth per warp (kStages-1 stages in flight while computing)
 constexpr int kStageBytes = kRows * (kSlots * 8 + 16);                  // 3328 B: values + index records
 constexpr int kRingBytes = kWarpsPerCta * kStages * kStageBytes;        // 159,744 B per CTA
 constexpr int kBarBytes = kWarpsPerCta * kStages * 8;                   // mbarriers

@@ -145,57 +145,76 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       : "memory");
 }
 
+// Per-warp ring state.  Stage counters advance incrementally (no div/mod); lane 0 owns the issue pointers.
 struct Ring {
   const unsigned char* base;  // generic address of this warp's stage 0
   uint32_t ring, bar;         // shared addresses of stage 0 and mbarrier 0
   int64_t r_lo, r_hi, nst;    // row range and number of stages
+  // consumer side
+  int slot;
+  uint32_t phase;
+  // producer side (lane 0)
+  int64_t issued;             // stages issued so far
+  int islot;
+  const double* vsrc;         // next stage's values
+  const IdxRec* isrc;         // next stage's index records
+  int64_t left;               // rows not yet issued
 };
 
-__device__ __forceinline__ Ring ring_setup(const SysView& S, unsigned char* dsm, int wid, int lane, int64_t r_lo,
-                                           int64_t r_hi) {
-  Ring R;
+__device__ __forceinline__ void ring_setup(Ring& R, const SysView& S, unsigned char* dsm, int wid, int lane,
+                                           int64_t r_lo, int64_t r_hi) {
   R.base = dsm + (size_t)wid * kStages * kStageBytes;
   R.ring = smem_u32(R.base);
   R.bar = smem_u32(dsm + kRingBytes) + wid * kStages * 8;
   R.r_lo = r_lo;
   R.r_hi = r_hi;
   R.nst = (r_hi - r_lo + kRows - 1) / kRows;
+  R.slot = 0;
+  R.phase = 0;
+  R.issued = 0;
+  R.islot = 0;
+  R.vsrc = S.vals + r_lo * kSlots;
+  R.isrc = S.idx + r_lo;
+  R.left = r_hi - r_lo;
   if (lane == 0) {
     for (int q = 0; q < kStages; ++q) mbar_init(R.bar + 8 * q, 1);
     fence_mbar_init();
   }
   __syncwarp();
-  return R;
 }
 
-__device__ __forceinline__ void ring_issue(const SysView& S, const Ring& R, int64_t k) {  // lane 0 only
-  const int slot = (int)(k % kStages);
-  const int64_t row0 = R.r_lo + k * kRows;
-  const uint32_t n = (uint32_t)min((int64_t)kRows, R.r_hi - row0);
-  const uint32_t bar = R.bar + 8 * slot, dst = R.ring + slot * kStageBytes;
+__device__ __forceinline__ void ring_issue(Ring& R) {  // lane 0 only
+  const uint32_t n = (uint32_t)(R.left < kRows ? R.left : kRows);
+  const uint32_t bar = R.bar + 8 * R.islot, dst = R.ring + R.islot * kStageBytes;
   mbar_expect_tx(bar, n * (kSlots * 8 + 16));
-  bulk_g2s(dst, S.vals + row0 * kSlots, n * kSlots * 8, bar);
-  bulk_g2s(dst + kRows * kSlots * 8, S.idx + row0, n * 16, bar);
+  bulk_g2s(dst, R.vsrc, n * (kSlots * 8), bar);
+  bulk_g2s(dst + kRows * kSlots * 8, R.isrc, n * 16, bar);
+  R.vsrc += kRows * kSlots;
+  R.isrc += kRows;
+  R.left -= n;
+  R.islot = R.islot + 1 == kStages ? 0 : R.islot + 1;
+  ++R.issued;
 }
 
-__device__ __forceinline__ void ring_prologue(const SysView& S, const Ring& R, int lane) {
+__device__ __forceinline__ void ring_prologue(Ring& R, int lane) {
   if (lane == 0)
-    for (int64_t k = 0; k < kStages && k < R.nst; ++k) ring_issue(S, R, k);
+    while (R.issued < kStages && R.issued < R.nst) ring_issue(R);
 }
 
-// after the warp has consumed stage k: refill its slot with stage k + kStages
-__device__ __forceinline__ void ring_release(const SysView& S, const Ring& R, int64_t k, int lane) {
+// after the warp has consumed the current stage: refill its slot with the next un-issued stage
+__device__ __forceinline__ void ring_release(Ring& R, int lane) {
   __syncwarp();
-  if (lane == 0 && k + kStages < R.nst) {
+  if (lane == 0 && R.issued < R.nst) {
     fence_proxy_async();
-    ring_issue(S, R, k + kStages);
+    ring_issue(R);
   }
+  R.slot = R.slot + 1 == kStages ? 0 : R.slot + 1;
+  R.phase ^= (R.slot == 0);
 }
 
-__device__ __forceinline__ const unsigned char* ring_wait(const Ring& R, int64_t k) {
-  const int slot = (int)(k % kStages);
-  mbar_wait(R.bar + 8 * slot, (uint32_t)((k / kStages) & 1));
-  return R.base + slot * kStageBytes;
+__device__ __forceinline__ const unsigned char* ring_wait(const Ring& R) {
+  mbar_wait(R.bar + 8 * R.slot, R.phase);
+  return R.base + R.slot * kStageBytes;
 }
 
 // row lr (0..kRows-1) of a stage: the lane's 6 values and the index record (16-B broadcast within the row group)
@@ -213,7 +232,7 @@ __device__ __forceinline__ void stage_row(const unsigned char* stg, int lr, int 
   rec.ic01 = (uint32_t)q.y; rec.ic23 = (uint32_t)q.z; rec.ic45 = (uint32_t)q.w;
 }
 
-// local column of the lane's slot t (t=5, j=3 is the global column; caller masks it when n_glob == 0)
+// local column of the lane's slot t (setup kernels only; the hot loops use hoisted pointers)
 __device__ __forceinline__ int64_t col_of(const SysView& S, int t, int j, int64_t star, const IdxRec& r) {
   if (t == 0) return 5 * star + j;
   if (t <= 3) return S.A0 + (int64_t)(t - 1) * S.n_axis + r.k0 + j;
@@ -222,11 +241,23 @@ __device__ __forceinline__ int64_t col_of(const SysView& S, int t, int j, int64_
 }
 
 // lane-local star of a row (rows are grouped by star, visited in increasing order): s / bound cached in registers
-__device__ __forceinline__ void track_star(const SysView& S, int64_t row, int64_t& s, int64_t& bound) {
+__device__ __forceinline__ bool track_star(const SysView& S, int64_t row, int64_t& s, int64_t& bound) {
+  bool moved = false;
   while (bound <= row) {
     ++s;
     bound = S.star_ptr[s + 1];
+    moved = true;
   }
+  return moved;
+}
+
+// instrumental index of the lane's t=5 slot (lanes 1, 2: instr 4, 5; others: 0, a safe dummy)
+__device__ __forceinline__ uint32_t ic5_of(const IdxRec& r, int j) {
+  return (j == 1) ? (r.ic45 & 0xffffu) : ((j == 2) ? (r.ic45 >> 16) : 0u);
+}
+__device__ __forceinline__ uint32_t ic4_of(const IdxRec& r, int j) {
+  const uint32_t w = j < 2 ? r.ic01 : r.ic23;
+  return (j & 1) ? (w >> 16) : (w & 0xffffu);
 }
 
 // ------------------------------------------------------------------------------------------------ aprod1
@@ -250,27 +281,31 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const double uscale = MODE == AP1_LSQR ? st->u_scale : 0.0;
   const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
-  const Ring R = ring_setup(S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
-  ring_prologue(S, R, lane);
-  const bool glob_ok = S.n_glob != 0;
+  Ring R;
+  ring_setup(R, S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
+  ring_prologue(R, lane);
+  // loop-invariant per-lane gather bases (32-bit offsets inside the loop)
+  const double* xatt0 = x + S.A0 + j;
+  const double* xatt1 = xatt0 + S.n_axis;
+  const double* xatt2 = xatt1 + S.n_axis;
+  const double* xins = SMEM_INSTR ? sh_x : x + S.I0;
+  const double vglob = S.n_glob ? __ldg(x + S.G0) : 0.0;
   int64_t s = s_lo, bound = S.star_ptr[s_lo + 1];
+  const double* xs = x + 5 * s_lo;
   double b2 = 0.0;
+  double* yp = y + R.r_lo + r;  // this lane's row in the current group
   double ynext[kGroups];
 #pragma unroll
-  for (int q = 0; q < kGroups; ++q) {
-    const int64_t row = R.r_lo + q * 8 + r;
-    ynext[q] = row < R.r_hi ? __ldg(y + row) : 0.0;
-  }
-  for (int64_t k = 0; k < R.nst; ++k) {
-    const int64_t row0 = R.r_lo + k * kRows;
+  for (int q = 0; q < kGroups; ++q) ynext[q] = (R.r_lo + q * 8 + r < R.r_hi) ? __ldg(yp + q * 8) : 0.0;
+  int64_t row0 = R.r_lo;
+  for (int64_t k = 0; k < R.nst; ++k, row0 += kRows, yp += kRows) {
     double ycur[kGroups];
 #pragma unroll
     for (int q = 0; q < kGroups; ++q) {  // prefetch next stage's y (u_hat)
       ycur[q] = ynext[q];
-      const int64_t row = row0 + kRows + q * 8 + r;
-      ynext[q] = row < R.r_hi ? __ldg(y + row) : 0.0;
+      ynext[q] = (row0 + kRows + q * 8 + r < R.r_hi) ? __ldg(yp + kRows + q * 8) : 0.0;
     }
-    const unsigned char* stg = ring_wait(R, k);
+    const unsigned char* stg = ring_wait(R);
     double v[kGroups][6], xv[kGroups][6];
     bool valid[kGroups];
 #pragma unroll
@@ -279,16 +314,23 @@ __global__ void __launch_bounds__(kThreads, 1)
       valid[q] = row < R.r_hi;
       IdxRec rec;
       stage_row(stg, q * 8 + r, j, v[q], rec);
-      if (valid[q]) track_star(S, row, s, bound);
+      if (valid[q]) {
+        if (track_star(S, row, s, bound)) xs = x + 5 * s;
+        const int k0 = rec.k0;
+        xv[q][0] = __ldg(xs + j);
+        xv[q][1] = __ldg(xatt0 + k0);
+        xv[q][2] = __ldg(xatt1 + k0);
+        xv[q][3] = __ldg(xatt2 + k0);
+        xv[q][4] = SMEM_INSTR ? xins[ic4_of(rec, j)] : __ldg(xins + ic4_of(rec, j));
+        const double a_ins = SMEM_INSTR ? xins[ic5_of(rec, j)] : __ldg(xins + ic5_of(rec, j));
+        const double a_ast = __ldg(xs + 4);
+        xv[q][5] = j == 0 ? a_ast : (j == 3 ? vglob : a_ins);
+      } else {
 #pragma unroll
-      for (int t = 0; t < 6; ++t) {
-        const bool ok = valid[q] && !(t == 5 && j == 3 && !glob_ok);
-        const bool in_smem = SMEM_INSTR && (t == 4 || (t == 5 && (j == 1 || j == 2)));
-        if (in_smem) xv[q][t] = ok ? sh_x[ic_of(rec, t == 4 ? j : 3 + j)] : 0.0;
-        else xv[q][t] = ok ? __ldg(x + col_of(S, t, j, s, rec)) : 0.0;
+        for (int t = 0; t < 6; ++t) xv[q][t] = 0.0;
       }
     }
-    ring_release(S, R, k, lane);
+    ring_release(R, lane);
 #pragma unroll
     for (int q = 0; q < kGroups; ++q) {
       double p = 0.0;
@@ -296,14 +338,13 @@ __global__ void __launch_bounds__(kThreads, 1)
       for (int t = 0; t < 6; ++t) p = fma(v[q][t], xv[q][t], p);
       p += __shfl_xor_sync(0xffffffffu, p, 1);
       p += __shfl_xor_sync(0xffffffffu, p, 2);
-      const int64_t row = row0 + q * 8 + r;
       if (valid[q] && j == 0) {
         if (MODE == AP1_LSQR) {
           const double un = p - uscale * ycur[q];
-          y[row] = un;
+          yp[q * 8] = un;
           b2 = fma(un, un, b2);
         } else {
-          y[row] = ycur[q] + p;
+          yp[q * 8] = ycur[q] + p;
         }
       }
     }
@@ -348,10 +389,13 @@ __global__ void __launch_bounds__(kThreads, 1)
   const double inv_beta = MODE == AP2_LSQR ? st->inv_beta : 1.0;
   const double beta = MODE == AP2_LSQR ? st->beta : 0.0;
   const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
-  const Ring R = ring_setup(S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
-  ring_prologue(S, R, lane);
+  Ring R;
+  ring_setup(R, S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
+  ring_prologue(R, lane);
   const bool glob_ok = S.n_glob != 0;
-  double* z_att = zsh;
+  double* zatt0 = zsh + j;
+  double* zatt1 = zatt0 + S.n_axis;
+  double* zatt2 = zatt1 + S.n_axis;
   double* z_ins = SMEM_INSTR ? sh_instr : zsh + S.n_att;
   double gacc = 0.0, a2 = 0.0, acc0 = 0.0, acc1 = 0.0;
   int64_t s = s_lo, bound = S.star_ptr[s_lo + 1];  // lane-local star of the lane's row
@@ -376,43 +420,41 @@ __global__ void __launch_bounds__(kThreads, 1)
           if (j == 0 && a == 4) z1 += c;
         }
       }
-      const int64_t c0 = 5 * star + j;
+      double* xc = xv + 5 * star;
       if (MODE == AP2_LSQR) {
-        const double vn = z0 - beta * xv[c0];
-        xv[c0] = vn;
+        const double vn = z0 - beta * xc[j];
+        xc[j] = vn;
         a2 = fma(vn, vn, a2);
         if (j == 0) {
-          const double vn1 = z1 - beta * xv[5 * star + 4];
-          xv[5 * star + 4] = vn1;
+          const double vn1 = z1 - beta * xc[4];
+          xc[4] = vn1;
           a2 = fma(vn1, vn1, a2);
         }
       } else if (MODE == AP2_PLAIN) {
-        xv[c0] += z0;
-        if (j == 0) xv[5 * star + 4] += z1;
+        xc[j] += z0;
+        if (j == 0) xc[4] += z1;
       } else {
-        xv[c0] = z0;
-        if (j == 0) xv[5 * star + 4] = z1;
+        xc[j] = z0;
+        if (j == 0) xc[4] = z1;
       }
     }
   };
 
   const double* ysrc = MODE == AP2_COLNORM ? nullptr : yv;
+  const double* yp = ysrc ? ysrc + R.r_lo + r : nullptr;
   double ynext[kGroups];
 #pragma unroll
-  for (int q = 0; q < kGroups; ++q) {
-    const int64_t row = R.r_lo + q * 8 + r;
-    ynext[q] = (ysrc && row < R.r_hi) ? __ldg(ysrc + row) : 0.0;
-  }
-  for (int64_t k = 0; k < R.nst; ++k) {
-    const int64_t row0 = R.r_lo + k * kRows;
+  for (int q = 0; q < kGroups; ++q) ynext[q] = (ysrc && R.r_lo + q * 8 + r < R.r_hi) ? __ldg(yp + q * 8) : 0.0;
+  int64_t row0 = R.r_lo;
+  for (int64_t k = 0; k < R.nst; ++k, row0 += kRows) {
     double ycur[kGroups];
 #pragma unroll
     for (int q = 0; q < kGroups; ++q) {
       ycur[q] = ynext[q];
-      const int64_t row = row0 + kRows + q * 8 + r;
-      ynext[q] = (ysrc && row < R.r_hi) ? __ldg(ysrc + row) : 0.0;
+      ynext[q] = (ysrc && row0 + kRows + q * 8 + r < R.r_hi) ? __ldg(yp + kRows + q * 8) : 0.0;
     }
-    const unsigned char* stg = ring_wait(R, k);
+    if (ysrc) yp += kRows;
+    const unsigned char* stg = ring_wait(R);
 #pragma unroll
     for (int q = 0; q < kGroups; ++q) {
       const int64_t base = row0 + q * 8;
@@ -428,12 +470,14 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (valid) {
         track_star(S, row, s, bound);
         // attitude: 3 axes x 4 consecutive knots -> sector-coalesced REDs (one per axis per lane)
-#pragma unroll
-        for (int t = 1; t <= 3; ++t) atomicAdd(z_att + (int64_t)(t - 1) * S.n_axis + rec.k0 + j, c[t]);
+        const int k0 = rec.k0;
+        atomicAdd(zatt0 + k0, c[1]);
+        atomicAdd(zatt1 + k0, c[2]);
+        atomicAdd(zatt2 + k0, c[3]);
         // instrumental
-        atomicAdd(z_ins + ic_of(rec, j), c[4]);
-        if (j == 1 || j == 2) atomicAdd(z_ins + ic_of(rec, 3 + j), c[5]);
-        if (j == 3 && glob_ok) gacc += c[5];
+        atomicAdd(z_ins + ic4_of(rec, j), c[4]);
+        if (j == 1 || j == 2) atomicAdd(z_ins + ic5_of(rec, j), c[5]);
+        if (j == 3) gacc += c[5];
       }
       // astrometric: segmented by star (rows are grouped by star)
       const double c0 = c[0], c5 = (j == 0) ? c[5] : 0.0;
@@ -453,7 +497,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
       }
     }
-    ring_release(S, R, k, lane);
+    ring_release(R, lane);
   }
   while (cs < s_hi) {  // empty trailing stars
     acc0 = 0.0; acc1 = 0.0;
