@@ -291,7 +291,12 @@ __global__ void __launch_bounds__(kThreads, 1)
   const double* xins = SMEM_INSTR ? sh_x : x + S.I0;
   const double vglob = S.n_glob ? __ldg(x + S.G0) : 0.0;
   int64_t s = s_lo, bound = S.star_ptr[s_lo + 1];
-  const double* xs = x + 5 * s_lo;
+  // the lane's astrometric values of its current star live in registers (reloaded only when the star changes)
+  double xa_j = 0.0, xa_4 = 0.0;
+  if (s_lo < s_hi) {
+    xa_j = __ldg(x + 5 * s_lo + j);
+    xa_4 = __ldg(x + 5 * s_lo + 4);
+  }
   double b2 = 0.0;
   double* yp = y + R.r_lo + r;  // this lane's row in the current group
   double ynext[kGroups];
@@ -314,21 +319,20 @@ __global__ void __launch_bounds__(kThreads, 1)
       valid[q] = row < R.r_hi;
       IdxRec rec;
       stage_row(stg, q * 8 + r, j, v[q], rec);
-      if (valid[q]) {
-        if (track_star(S, row, s, bound)) xs = x + 5 * s;
-        const int k0 = rec.k0;
-        xv[q][0] = __ldg(xs + j);
-        xv[q][1] = __ldg(xatt0 + k0);
-        xv[q][2] = __ldg(xatt1 + k0);
-        xv[q][3] = __ldg(xatt2 + k0);
-        xv[q][4] = SMEM_INSTR ? xins[ic4_of(rec, j)] : __ldg(xins + ic4_of(rec, j));
-        const double a_ins = SMEM_INSTR ? xins[ic5_of(rec, j)] : __ldg(xins + ic5_of(rec, j));
-        const double a_ast = __ldg(xs + 4);
-        xv[q][5] = j == 0 ? a_ast : (j == 3 ? vglob : a_ins);
-      } else {
-#pragma unroll
-        for (int t = 0; t < 6; ++t) xv[q][t] = 0.0;
+      if (valid[q] && track_star(S, row, s, bound)) {
+        xa_j = __ldg(x + 5 * s + j);
+        xa_4 = __ldg(x + 5 * s + 4);
       }
+      // only the attitude values are gathered from global memory (L2) per row; instr from shared memory
+      const int k0 = valid[q] ? rec.k0 : 0;
+      xv[q][0] = xa_j;
+      xv[q][1] = __ldg(xatt0 + k0);
+      xv[q][2] = __ldg(xatt1 + k0);
+      xv[q][3] = __ldg(xatt2 + k0);
+      const uint32_t i4 = valid[q] ? ic4_of(rec, j) : 0u, i5 = valid[q] ? ic5_of(rec, j) : 0u;
+      xv[q][4] = SMEM_INSTR ? xins[i4] : __ldg(xins + i4);
+      const double a_ins = SMEM_INSTR ? xins[i5] : __ldg(xins + i5);
+      xv[q][5] = j == 0 ? xa_4 : (j == 3 ? vglob : a_ins);
     }
     ring_release(R, lane);
 #pragma unroll

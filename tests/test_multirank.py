@@ -133,7 +133,7 @@ def _gpu_worker(rank, world, port, q, itn):
 def test_gpu_two_rank_lsqr_matches_single_rank(cuda_device):
     import torch
     import paper_conf_sc_malenzacsbvba24_b200 as avu
-    itn = 100  # converged (x parity needs convergence, SURVEY EXP-3)
+    itn = 160  # converged (x parity needs convergence, SURVEY EXP-3)
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
