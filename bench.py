@@ -242,7 +242,7 @@ def run_ours(args):
         se.set_system_ptrs(pin["vals"].data_ptr(), pin["mA"].data_ptr(), pin["mT"].data_ptr(),
                            pin["iC"].data_ptr(), pin["b"].data_ptr())
         se.precondition()
-        r = se.solve(x_out=xo, se_out=so, itn_limit=K, atol=0, btol=0, conlim=0, fixed_count=True)
+        r = se.solve(x_out=xo, se_out=so, itn_limit=K, atol=0, btol=0, conlim=0, fixed_count=True, fused=args.fused)
         barrier()
         t_e2e = max_over_ranks(time.perf_counter() - t0)
         h2d = sum(t.numel() * t.element_size() for t in pin.values())
@@ -258,7 +258,7 @@ def run_ours(args):
     s = avu.Solver.synthetic(w, rank=rank, nranks=world, **kw)
     t0 = time.perf_counter()
     s.precondition()
-    s.init(itn_limit=K + Wm + 10, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=False)
+    s.init(itn_limit=K + Wm + 10, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=False, fused=args.fused)
     s.sync()
     t_setup = time.perf_counter() - t0
     if Wm > 0:
@@ -274,7 +274,15 @@ def run_ours(args):
     peak, peak_kind = measured_peaks()
     ap1_b, ap2_b, it_b = algorithmic_bytes(w, s.n_local_rows, s.star_end - s.star_begin, s.n_shared,
                                            s.n_local_cols)
-    if ap2_ms >= ap1_ms:
+    if args.fused:
+        # fused single pass (NEXT-1): A, indices, u_hat read once + u_hat written (224 B/row), v_astro read and
+        # zA written (80 B/star), v_shared gathered and z_shared written once (16 B/column)
+        n_st = s.star_end - s.star_begin
+        fz_b = 224 * s.n_local_rows + 80 * n_st + 16 * s.n_shared
+        it_b = 224 * s.n_local_rows + 56 * s.n_local_cols + 80 * n_st
+        kname, kb, kms = "fused", fz_b, ap1_ms
+        ap1_b = fz_b
+    elif ap2_ms >= ap1_ms:
         kname, kb, kms = "aprod2", ap2_b, ap2_ms
     else:
         kname, kb, kms = "aprod1", ap1_b, ap1_ms
@@ -293,7 +301,10 @@ def run_ours(args):
                                "frac": round(it_b / (ms_step * 1e-3) / 1e9 / peak, 4),
                                "aprod1_ms": round(ap1_ms, 4), "aprod2_ms": round(ap2_ms, 4),
                                "aprod1_frac": round(ap1_b / (ap1_ms * 1e-3) / 1e9 / peak, 4),
-                               "aprod2_frac": round(ap2_b / (ap2_ms * 1e-3) / 1e9 / peak, 4)},
+                               "aprod2_frac": (round(ap2_b / (ap2_ms * 1e-3) / 1e9 / peak, 4)
+                                               if not args.fused else None),
+                               "variant": "fused single pass (SURVEY 8(f) NEXT-1; bytes are its own 224 B/row)"
+                               if args.fused else "two-pass (SURVEY 8(a)); 440 B/row"},
         "gpu_launches": int(max_over_ranks(r["launches"])),
         "clocks": clk.summary(),
         "e2e": e2e,
@@ -320,6 +331,7 @@ def main():
     ap.add_argument("--no-e2e", dest="e2e", action="store_false")
     ap.add_argument("--no-cpu-baseline", dest="cpu_baseline", action="store_false")
     ap.add_argument("--cpu-iters", type=int, default=3)
+    ap.add_argument("--fused", action="store_true", help="fused single-pass iteration (SURVEY 8(f) NEXT-1)")
     args = ap.parse_args()
     if args.warmup < 3:
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)

@@ -108,8 +108,9 @@ typedef struct {
                               P:L1763-1767); the first nonzero istop is reported in istop_first */
   int32_t use_graph;       /* 1: replay the iteration as a CUDA graph (default for small systems) */
   int32_t poll_every;      /* host polls the stop flag every k iterations (<= 0 => 16) */
-  int32_t fused;           /* 0: two-pass iteration (aprod1 then aprod2; default).  1: reserved (fused single
-                              pass) */
+  int32_t fused;           /* 0: two-pass iteration (aprod1 then aprod2; default).  1: fused single pass
+                              (SURVEY §8(f) NEXT-1): u_hat = A v - (alpha/beta) u_hat and z = A^T u_hat in ONE read
+                              of A, then v' = z/beta - beta v; same results up to rounding */
 } lsqr_solve_params;
 
 typedef struct {
@@ -204,8 +205,9 @@ int lsqr_solve(lsqr_t h, const lsqr_solve_params* p, lsqr_result* res, double* x
 int lsqr_init(lsqr_t h, const lsqr_solve_params* p);
 int lsqr_iterate(lsqr_t h, int64_t n_iter);
 /* n_iter iterations without graph replay, with CUDA events around every kernel launch on the launching stream.
- * out[0] = total ms, out[1] = sum of aprod1 kernel ms, out[2] = sum of aprod2 kernel ms, out[3] = kernels launched,
- * out[4] = ms of the slowest single iteration.  Synchronous. */
+ * out[0] = total ms, out[1] = sum of aprod1 kernel ms (fused mode: the fused row kernel), out[2] = sum of aprod2
+ * kernel ms (fused mode: the astro column pass), out[3] = kernels launched, out[4] = ms of the slowest single
+ * iteration.  Synchronous. */
 int lsqr_iterate_timed(lsqr_t h, int64_t n_iter, double* out);
 int lsqr_finalize(lsqr_t h, lsqr_result* res, double* x_out, double* se_out);
 /* State snapshot (host pointers, any may be NULL; synchronous): scalars [LSQR_NSCALARS]; u [n_local_rows+n_constr]

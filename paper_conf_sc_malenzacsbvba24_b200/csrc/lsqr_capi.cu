@@ -93,6 +93,7 @@ struct lsqr_ctx {
   std::vector<void*> allocs;
   double *vals = nullptr, *u = nullptr, *v = nullptr, *w = nullptr, *x = nullptr, *var = nullptr, *D = nullptr;
   double *zsh = nullptr, *part_rows = nullptr, *part_a2 = nullptr, *cpart = nullptr, *part_sh = nullptr;
+  double *zA = nullptr, *part_va = nullptr;  // fused mode: astro z (A^T u_hat) and alpha^2 partials of k_vastro
   double *part_wa = nullptr, *part_ws = nullptr, *part_g1 = nullptr, *ar1 = nullptr, *uc = nullptr,
          *ucn = nullptr, *crhs = nullptr, *tmp = nullptr, *tmax = nullptr;
   IdxRec* idx = nullptr;
@@ -240,8 +241,13 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   SysView& S = h->S;
   cudaStream_t s = h->s;
   const bool multi = h->nranks > 1;
+  const bool fused = h->params.fused != 0;
   if (ev) cudaEventRecord(ev[0], s);
-  CKL(h, launch_aprod1(AP1_LSQR, S, h->grid, h->v, h->u, h->part_rows, h->cpart, h->st, s), "aprod1");
+  if (fused) {  // NEXT-1: u_hat update and A^T u_hat in one read of A
+    CKL(h, launch_fused(S, h->grid, h->v, h->u, h->zA, h->zsh, h->part_rows, h->cpart, h->st, s), "fused");
+  } else {
+    CKL(h, launch_aprod1(AP1_LSQR, S, h->grid, h->v, h->u, h->part_rows, h->cpart, h->st, s), "aprod1");
+  }
   if (ev) cudaEventRecord(ev[1], s);
   if (!multi) {
     CKL(h, launch_beta(0, S, h->part_rows, h->W, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta");
@@ -253,16 +259,26 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
     CKL(h, launch_beta(2, S, h->part_rows, h->W, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta2");
   }
   if (ev) cudaEventRecord(ev[2], s);
-  CKL(h, launch_aprod2(AP2_LSQR, S, h->grid, h->u, h->ucn, h->v, h->zsh, h->part_a2, h->st, h->rank == 0, s),
-      "aprod2");
+  const double* a2part;
+  int64_t n_a2;
+  if (fused) {
+    CKL(h, launch_vastro(S, h->v, h->zA, h->uc, h->zsh, h->part_va, kG3, h->st, h->rank == 0, s), "vastro");
+    a2part = h->part_va;
+    n_a2 = kG3;
+  } else {
+    CKL(h, launch_aprod2(AP2_LSQR, S, h->grid, h->u, h->ucn, h->v, h->zsh, h->part_a2, h->st, h->rank == 0, s),
+        "aprod2");
+    a2part = h->part_a2;
+    n_a2 = h->W;
+  }
   if (ev) cudaEventRecord(ev[3], s);
   if (multi) {
     // AR2 payload: [z_att | z_instr | z_glob | alpha^2 astro local]
-    CKL(h, launch_sum_to(h->part_a2, h->W, h->zsh + h->n_sh, s), "a2sum");
+    CKL(h, launch_sum_to(a2part, n_a2, h->zsh + h->n_sh, s), "a2sum");
     CKR(allreduce(h, h->zsh, h->n_sh + 1));
   }
-  CKL(h, launch_vshared(S, h->v + S.A0, h->zsh, h->part_sh, kG2, h->st, s), "vshared");
-  CKL(h, launch_scalar(h->st, h->part_a2, h->W, h->part_sh, kG2, h->part_wa, kG3, h->part_ws, kG3,
+  CKL(h, launch_vshared(S, h->v + S.A0, h->zsh, h->part_sh, kG2, h->st, fused ? 1 : 0, s), "vshared");
+  CKL(h, launch_scalar(h->st, a2part, n_a2, h->part_sh, kG2, h->part_wa, kG3, h->part_ws, kG3,
                        multi ? h->zsh + h->n_sh : nullptr, multi ? h->ar1 + h->n_constr + 1 : nullptr, 0,
                        h->hflag_dev, s),
       "scalar");
@@ -271,7 +287,7 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   return LSQR_OK;
 }
 
-int kernels_per_iteration(lsqr_t h) { return h->nranks > 1 ? 9 : 6; }
+int kernels_per_iteration(lsqr_t h) { return h->nranks > 1 ? 9 : 6; }  // same count in both modes
 
 int build_graph(lsqr_t h) {
   if (h->gexec) {
@@ -549,6 +565,8 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   AL(h->part_a2, h->W);
   AL(h->cpart, std::max<int64_t>((int64_t)ch_row.size(), 1));
   AL(h->part_sh, kG2);
+  AL(h->zA, 5 * h->n_loc_stars);
+  AL(h->part_va, kG3);
   AL(h->part_wa, kG3);
   AL(h->part_ws, kG3);
   AL(h->part_g1, kG1);
@@ -847,7 +865,7 @@ int lsqr_init(lsqr_t h, const lsqr_solve_params* p) {
     CKL(h, launch_sum_to(h->part_a2, h->W, h->zsh + h->n_sh, h->s), "a2sum");
     CKR(allreduce(h, h->zsh, h->n_sh + 1));
   }
-  CKL(h, launch_vshared(S, h->v + S.A0, h->zsh, h->part_sh, kG2, h->st, h->s), "vshared");
+  CKL(h, launch_vshared(S, h->v + S.A0, h->zsh, h->part_sh, kG2, h->st, 0, h->s), "vshared");
   CKL(h, launch_scalar(h->st, h->part_a2, h->W, h->part_sh, kG2, h->part_wa, kG3, h->part_ws, kG3,
                        multi ? h->zsh + h->n_sh : nullptr, nullptr, 1, h->hflag_dev, h->s),
       "scalar0");

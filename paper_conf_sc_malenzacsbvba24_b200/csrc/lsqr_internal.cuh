@@ -101,7 +101,12 @@ cudaError_t launch_beta(int phase, const SysView& S, const double* part, int64_t
                         cudaStream_t s);
 cudaError_t launch_cdot_add(const SysView& S, const double* cpart, const double* ar1, double* yc, cudaStream_t s);
 cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* part, int nblk, const DevState* st,
-                           cudaStream_t s);
+                           int fused, cudaStream_t s);
+// NEXT-1 fused single pass (u_hat update + A^T u_hat in one read of A) and its astro column pass
+cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh,
+                         double* part, double* cpart, const DevState* st, cudaStream_t s);
+cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const double* uc, double* zsh, double* part,
+                          int nblk, const DevState* st, int do_shared_constr, cudaStream_t s);
 cudaError_t launch_add_shared(double* xsh, double* zsh, int64_t n, int mode, cudaStream_t s);
 cudaError_t launch_scalar(DevState* st, const double* part_astro, int64_t n_pa, const double* part_sh,
                           int64_t n_ps, const double* part_wa, int64_t n_pwa, const double* part_ws, int64_t n_pws,

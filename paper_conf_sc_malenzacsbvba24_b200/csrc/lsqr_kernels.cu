@@ -145,79 +145,81 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
       : "memory");
 }
 
-// Per-warp ring state.  Stage counters advance incrementally (no div/mod); lane 0 owns the issue pointers.
-struct Ring {
+// Per-warp ring state, templated on rows per stage and ring depth.  Stage counters advance incrementally (no
+// div/mod); lane 0 owns the issue pointers.
+template <int ROWS, int STAGES>
+struct RingT {
+  static constexpr int kStage = ROWS * (kSlots * 8 + 16);
+  static constexpr int kBytes = kWarpsPerCta * STAGES * kStage;
+  static constexpr int kBars = kWarpsPerCta * STAGES * 8;
   const unsigned char* base;  // generic address of this warp's stage 0
   uint32_t ring, bar;         // shared addresses of stage 0 and mbarrier 0
   int64_t r_lo, r_hi, nst;    // row range and number of stages
-  // consumer side
-  int slot;
+  int slot;                   // consumer side
   uint32_t phase;
-  // producer side (lane 0)
-  int64_t issued;             // stages issued so far
+  int64_t issued;             // producer side (lane 0)
   int islot;
-  const double* vsrc;         // next stage's values
-  const IdxRec* isrc;         // next stage's index records
-  int64_t left;               // rows not yet issued
+  const double* vsrc;
+  const IdxRec* isrc;
+  int64_t left;
+
+  __device__ __forceinline__ void setup(const SysView& S, unsigned char* dsm, int wid, int lane, int64_t lo,
+                                        int64_t hi) {
+    base = dsm + (size_t)wid * STAGES * kStage;
+    ring = smem_u32(base);
+    bar = smem_u32(dsm + kBytes) + wid * STAGES * 8;
+    r_lo = lo;
+    r_hi = hi;
+    nst = (hi - lo + ROWS - 1) / ROWS;
+    slot = 0;
+    phase = 0;
+    issued = 0;
+    islot = 0;
+    vsrc = S.vals + lo * kSlots;
+    isrc = S.idx + lo;
+    left = hi - lo;
+    if (lane == 0) {
+      for (int q = 0; q < STAGES; ++q) mbar_init(bar + 8 * q, 1);
+      fence_mbar_init();
+    }
+    __syncwarp();
+  }
+  __device__ __forceinline__ void issue() {  // lane 0 only
+    const uint32_t n = (uint32_t)(left < ROWS ? left : ROWS);
+    const uint32_t b = bar + 8 * islot, dst = ring + islot * kStage;
+    mbar_expect_tx(b, n * (kSlots * 8 + 16));
+    bulk_g2s(dst, vsrc, n * (kSlots * 8), b);
+    bulk_g2s(dst + ROWS * kSlots * 8, isrc, n * 16, b);
+    vsrc += ROWS * kSlots;
+    isrc += ROWS;
+    left -= n;
+    islot = islot + 1 == STAGES ? 0 : islot + 1;
+    ++issued;
+  }
+  __device__ __forceinline__ void prologue(int lane) {
+    if (lane == 0)
+      while (issued < STAGES && issued < nst) issue();
+  }
+  // after the warp has consumed the current stage: refill its slot with the next un-issued stage
+  __device__ __forceinline__ void release(int lane) {
+    __syncwarp();
+    if (lane == 0 && issued < nst) {
+      fence_proxy_async();
+      issue();
+    }
+    slot = slot + 1 == STAGES ? 0 : slot + 1;
+    phase ^= (slot == 0);
+  }
+  __device__ __forceinline__ const unsigned char* wait() const {
+    mbar_wait(bar + 8 * slot, phase);
+    return base + slot * kStage;
+  }
 };
-
-__device__ __forceinline__ void ring_setup(Ring& R, const SysView& S, unsigned char* dsm, int wid, int lane,
-                                           int64_t r_lo, int64_t r_hi) {
-  R.base = dsm + (size_t)wid * kStages * kStageBytes;
-  R.ring = smem_u32(R.base);
-  R.bar = smem_u32(dsm + kRingBytes) + wid * kStages * 8;
-  R.r_lo = r_lo;
-  R.r_hi = r_hi;
-  R.nst = (r_hi - r_lo + kRows - 1) / kRows;
-  R.slot = 0;
-  R.phase = 0;
-  R.issued = 0;
-  R.islot = 0;
-  R.vsrc = S.vals + r_lo * kSlots;
-  R.isrc = S.idx + r_lo;
-  R.left = r_hi - r_lo;
-  if (lane == 0) {
-    for (int q = 0; q < kStages; ++q) mbar_init(R.bar + 8 * q, 1);
-    fence_mbar_init();
-  }
-  __syncwarp();
-}
-
-__device__ __forceinline__ void ring_issue(Ring& R) {  // lane 0 only
-  const uint32_t n = (uint32_t)(R.left < kRows ? R.left : kRows);
-  const uint32_t bar = R.bar + 8 * R.islot, dst = R.ring + R.islot * kStageBytes;
-  mbar_expect_tx(bar, n * (kSlots * 8 + 16));
-  bulk_g2s(dst, R.vsrc, n * (kSlots * 8), bar);
-  bulk_g2s(dst + kRows * kSlots * 8, R.isrc, n * 16, bar);
-  R.vsrc += kRows * kSlots;
-  R.isrc += kRows;
-  R.left -= n;
-  R.islot = R.islot + 1 == kStages ? 0 : R.islot + 1;
-  ++R.issued;
-}
-
-__device__ __forceinline__ void ring_prologue(Ring& R, int lane) {
-  if (lane == 0)
-    while (R.issued < kStages && R.issued < R.nst) ring_issue(R);
-}
-
-// after the warp has consumed the current stage: refill its slot with the next un-issued stage
-__device__ __forceinline__ void ring_release(Ring& R, int lane) {
-  __syncwarp();
-  if (lane == 0 && R.issued < R.nst) {
-    fence_proxy_async();
-    ring_issue(R);
-  }
-  R.slot = R.slot + 1 == kStages ? 0 : R.slot + 1;
-  R.phase ^= (R.slot == 0);
-}
-
-__device__ __forceinline__ const unsigned char* ring_wait(const Ring& R) {
-  mbar_wait(R.bar + 8 * R.slot, R.phase);
-  return R.base + R.slot * kStageBytes;
-}
+using Ring = RingT<kRows, kStages>;
+static_assert(Ring::kBytes == kRingBytes && Ring::kBars == kBarBytes, "ring geometry");
 
 // row lr (0..kRows-1) of a stage: the lane's 6 values and the index record (16-B broadcast within the row group)
+template <int ROWS = kRows>
 __device__ __forceinline__ void stage_row(const unsigned char* stg, int lr, int j, double (&v)[6], IdxRec& rec) {
   // lane-major row: the lane's 6 values are 48 contiguous bytes -> three conflict-free 16-B shared loads
   const double2* rp = reinterpret_cast<const double2*>(stg + lr * kSlots * 8 + 48 * j);
@@ -227,7 +229,7 @@ __device__ __forceinline__ void stage_row(const unsigned char* stg, int lr, int 
     v[2 * q] = d.x;
     v[2 * q + 1] = d.y;
   }
-  const int4 q = *reinterpret_cast<const int4*>(stg + kRows * kSlots * 8 + lr * 16);
+  const int4 q = *reinterpret_cast<const int4*>(stg + ROWS * kSlots * 8 + lr * 16);
   rec.k0 = q.x;
   rec.ic01 = (uint32_t)q.y; rec.ic23 = (uint32_t)q.z; rec.ic45 = (uint32_t)q.w;
 }
@@ -251,13 +253,57 @@ __device__ __forceinline__ bool track_star(const SysView& S, int64_t row, int64_
   return moved;
 }
 
-// instrumental index of the lane's t=5 slot (lanes 1, 2: instr 4, 5; others: 0, a safe dummy)
-__device__ __forceinline__ uint32_t ic5_of(const IdxRec& r, int j) {
-  return (j == 1) ? (r.ic45 & 0xffffu) : ((j == 2) ? (r.ic45 >> 16) : 0u);
-}
+// instrumental index of the lane's t=5 slot: lanes 1, 2 -> instr 4, 5 (lanes 0, 3 get a harmless in-range dummy)
+__device__ __forceinline__ uint32_t ic5_of(const IdxRec& r, int j) { return (r.ic45 >> ((j & 2) << 3)) & 0xffffu; }
+// instrumental index of the lane's t=4 slot: instr j
 __device__ __forceinline__ uint32_t ic4_of(const IdxRec& r, int j) {
-  const uint32_t w = j < 2 ? r.ic01 : r.ic23;
-  return (j & 1) ? (w >> 16) : (w & 0xffffu);
+  const uint32_t w = (j & 2) ? r.ic23 : r.ic01;
+  return (w >> ((j & 1) << 4)) & 0xffffu;
+}
+
+// Astro values of the lane's current star in registers, with the NEXT star's values prefetched one star ahead so
+// a star change (every ~100-200 rows) does not stall the warp on a memory round trip.
+struct AstroCache {
+  double cj, c4, nj, n4;  // current / next star: x[5s+j], x[5s+4]
+  int64_t s;              // current star
+  __device__ __forceinline__ void init(const double* __restrict__ x, int64_t s0, int64_t s_hi, int j) {
+    s = s0;
+    cj = c4 = nj = n4 = 0.0;
+    if (s0 < s_hi) { cj = __ldg(x + 5 * s0 + j); c4 = __ldg(x + 5 * s0 + 4); }
+    if (s0 + 1 < s_hi) { nj = __ldg(x + 5 * (s0 + 1) + j); n4 = __ldg(x + 5 * (s0 + 1) + 4); }
+  }
+  __device__ __forceinline__ void move_to(const double* __restrict__ x, int64_t ns, int64_t s_hi, int j) {
+    if (ns == s + 1) { cj = nj; c4 = n4; }
+    else { cj = __ldg(x + 5 * ns + j); c4 = __ldg(x + 5 * ns + 4); }
+    s = ns;
+    if (ns + 1 < s_hi) { nj = __ldg(x + 5 * (ns + 1) + j); n4 = __ldg(x + 5 * (ns + 1) + 4); }
+  }
+};
+// Shared-memory FP64 accumulation of up to N independent (address, value) pairs with interleaved CAS retries
+// (sm_100a has no native shared-memory FP64 add; one CAS loop per update would serialise N round trips).
+template <int N>
+__device__ __forceinline__ void smem_add_n(double* const (&a)[N], const double (&val)[N], const bool (&on)[N]) {
+  unsigned long long old[N];
+  bool pend[N];
+#pragma unroll
+  for (int i = 0; i < N; ++i) {
+    pend[i] = on[i];
+    old[i] = pend[i] ? *reinterpret_cast<volatile unsigned long long*>(a[i]) : 0ull;
+  }
+  while (true) {
+    bool any = false;
+#pragma unroll
+    for (int i = 0; i < N; ++i) {
+      if (pend[i]) {
+        const unsigned long long nw = __double_as_longlong(__longlong_as_double(old[i]) + val[i]);
+        const unsigned long long got = atomicCAS(reinterpret_cast<unsigned long long*>(a[i]), old[i], nw);
+        pend[i] = got != old[i];
+        old[i] = got;
+        any |= pend[i];
+      }
+    }
+    if (!any) break;
+  }
 }
 
 // ------------------------------------------------------------------------------------------------ aprod1
@@ -282,8 +328,8 @@ __global__ void __launch_bounds__(kThreads, 1)
   const double uscale = MODE == AP1_LSQR ? st->u_scale : 0.0;
   const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
   Ring R;
-  ring_setup(R, S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
-  ring_prologue(R, lane);
+  R.setup(S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
+  R.prologue(lane);
   // loop-invariant per-lane gather bases (32-bit offsets inside the loop)
   const double* xatt0 = x + S.A0 + j;
   const double* xatt1 = xatt0 + S.n_axis;
@@ -291,12 +337,8 @@ __global__ void __launch_bounds__(kThreads, 1)
   const double* xins = SMEM_INSTR ? sh_x : x + S.I0;
   const double vglob = S.n_glob ? __ldg(x + S.G0) : 0.0;
   int64_t s = s_lo, bound = S.star_ptr[s_lo + 1];
-  // the lane's astrometric values of its current star live in registers (reloaded only when the star changes)
-  double xa_j = 0.0, xa_4 = 0.0;
-  if (s_lo < s_hi) {
-    xa_j = __ldg(x + 5 * s_lo + j);
-    xa_4 = __ldg(x + 5 * s_lo + 4);
-  }
+  AstroCache ac;  // the lane's astrometric values of its current (and next) star live in registers
+  ac.init(x, s_lo, s_hi, j);
   double b2 = 0.0;
   double* yp = y + R.r_lo + r;  // this lane's row in the current group
   double ynext[kGroups];
@@ -310,7 +352,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       ycur[q] = ynext[q];
       ynext[q] = (row0 + kRows + q * 8 + r < R.r_hi) ? __ldg(yp + kRows + q * 8) : 0.0;
     }
-    const unsigned char* stg = ring_wait(R);
+    const unsigned char* stg = R.wait();
     double v[kGroups][6], xv[kGroups][6];
     bool valid[kGroups];
 #pragma unroll
@@ -319,22 +361,19 @@ __global__ void __launch_bounds__(kThreads, 1)
       valid[q] = row < R.r_hi;
       IdxRec rec;
       stage_row(stg, q * 8 + r, j, v[q], rec);
-      if (valid[q] && track_star(S, row, s, bound)) {
-        xa_j = __ldg(x + 5 * s + j);
-        xa_4 = __ldg(x + 5 * s + 4);
-      }
+      if (valid[q] && track_star(S, row, s, bound)) ac.move_to(x, s, s_hi, j);
       // only the attitude values are gathered from global memory (L2) per row; instr from shared memory
       const int k0 = valid[q] ? rec.k0 : 0;
-      xv[q][0] = xa_j;
+      xv[q][0] = ac.cj;
       xv[q][1] = __ldg(xatt0 + k0);
       xv[q][2] = __ldg(xatt1 + k0);
       xv[q][3] = __ldg(xatt2 + k0);
       const uint32_t i4 = valid[q] ? ic4_of(rec, j) : 0u, i5 = valid[q] ? ic5_of(rec, j) : 0u;
       xv[q][4] = SMEM_INSTR ? xins[i4] : __ldg(xins + i4);
       const double a_ins = SMEM_INSTR ? xins[i5] : __ldg(xins + i5);
-      xv[q][5] = j == 0 ? xa_4 : (j == 3 ? vglob : a_ins);
+      xv[q][5] = j == 0 ? ac.c4 : (j == 3 ? vglob : a_ins);
     }
-    ring_release(R, lane);
+    R.release(lane);
 #pragma unroll
     for (int q = 0; q < kGroups; ++q) {
       double p = 0.0;
@@ -394,8 +433,8 @@ __global__ void __launch_bounds__(kThreads, 1)
   const double beta = MODE == AP2_LSQR ? st->beta : 0.0;
   const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
   Ring R;
-  ring_setup(R, S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
-  ring_prologue(R, lane);
+  R.setup(S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
+  R.prologue(lane);
   const bool glob_ok = S.n_glob != 0;
   double* zatt0 = zsh + j;
   double* zatt1 = zatt0 + S.n_axis;
@@ -405,6 +444,15 @@ __global__ void __launch_bounds__(kThreads, 1)
   int64_t s = s_lo, bound = S.star_ptr[s_lo + 1];  // lane-local star of the lane's row
   int64_t cs = s_lo;                                // warp-uniform star being accumulated
   int64_t cs_end = (cs < s_hi) ? S.star_ptr[cs + 1] : 0;
+  // old astro values of star cs, loaded when cs becomes current so the finalize does not wait on memory
+  double xo_j = 0.0, xo_4 = 0.0;
+  auto prefetch_old = [&](int64_t star) {
+    if (MODE != AP2_COLNORM && star < s_hi && lane < 4) {
+      xo_j = xv[5 * star + j];
+      xo_4 = xv[5 * star + 4];
+    }
+  };
+  prefetch_old(cs);
 
   auto finalize = [&](int64_t star) {
     double z0 = acc0, z1 = acc1;
@@ -426,17 +474,17 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       double* xc = xv + 5 * star;
       if (MODE == AP2_LSQR) {
-        const double vn = z0 - beta * xc[j];
+        const double vn = z0 - beta * xo_j;
         xc[j] = vn;
         a2 = fma(vn, vn, a2);
         if (j == 0) {
-          const double vn1 = z1 - beta * xc[4];
+          const double vn1 = z1 - beta * xo_4;
           xc[4] = vn1;
           a2 = fma(vn1, vn1, a2);
         }
       } else if (MODE == AP2_PLAIN) {
-        xc[j] += z0;
-        if (j == 0) xc[4] += z1;
+        xc[j] = xo_j + z0;
+        if (j == 0) xc[4] = xo_4 + z1;
       } else {
         xc[j] = z0;
         if (j == 0) xc[4] = z1;
@@ -458,7 +506,12 @@ __global__ void __launch_bounds__(kThreads, 1)
       ynext[q] = (ysrc && row0 + kRows + q * 8 + r < R.r_hi) ? __ldg(yp + kRows + q * 8) : 0.0;
     }
     if (ysrc) yp += kRows;
-    const unsigned char* stg = ring_wait(R);
+    const unsigned char* stg = R.wait();
+    double* ia[2 * kGroups];
+    double iv[2 * kGroups];
+    bool ion[2 * kGroups];
+#pragma unroll
+    for (int i = 0; i < 2 * kGroups; ++i) { ia[i] = z_ins; iv[i] = 0.0; ion[i] = false; }
 #pragma unroll
     for (int q = 0; q < kGroups; ++q) {
       const int64_t base = row0 + q * 8;
@@ -478,9 +531,18 @@ __global__ void __launch_bounds__(kThreads, 1)
         atomicAdd(zatt0 + k0, c[1]);
         atomicAdd(zatt1 + k0, c[2]);
         atomicAdd(zatt2 + k0, c[3]);
-        // instrumental
-        atomicAdd(z_ins + ic4_of(rec, j), c[4]);
-        if (j == 1 || j == 2) atomicAdd(z_ins + ic5_of(rec, j), c[5]);
+        // instrumental: collected for the whole stage, accumulated below with interleaved CAS (smem path)
+        if (SMEM_INSTR) {
+          ia[2 * q] = z_ins + ic4_of(rec, j);
+          iv[2 * q] = c[4];
+          ion[2 * q] = true;
+          ia[2 * q + 1] = z_ins + ic5_of(rec, j);
+          iv[2 * q + 1] = c[5];
+          ion[2 * q + 1] = (j == 1 || j == 2);
+        } else {
+          atomicAdd(z_ins + ic4_of(rec, j), c[4]);
+          if (j == 1 || j == 2) atomicAdd(z_ins + ic5_of(rec, j), c[5]);
+        }
         if (j == 3) gacc += c[5];
       }
       // astrometric: segmented by star (rows are grouped by star)
@@ -495,18 +557,21 @@ __global__ void __launch_bounds__(kThreads, 1)
             ++cs;
             if (cs >= s_hi) break;
             cs_end = S.star_ptr[cs + 1];
+            prefetch_old(cs);
           } else {
             break;
           }
         }
       }
     }
-    ring_release(R, lane);
+    if (SMEM_INSTR) smem_add_n<2 * kGroups>(ia, iv, ion);
+    R.release(lane);
   }
   while (cs < s_hi) {  // empty trailing stars
     acc0 = 0.0; acc1 = 0.0;
     finalize(cs);
     ++cs;
+    prefetch_old(cs);
   }
   // global column: one RED per warp
   if (glob_ok) {
@@ -532,6 +597,203 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (v != 0.0) atomicAdd(zsh + S.n_att + i, v);
     }
   }
+}
+
+
+// ------------------------------------------------------------------------------------------------ fused pass
+// NEXT-1: one pass over the rows per iteration.  For each row
+//     u_hat_i = a_i . v - u_scale * u_hat_i          (aprod1, Paige-Saunders step a)
+//     z      += a_i^T u_hat_i                         (aprod2 with the UNNORMALISED new u; beta is not known yet)
+// so A is read once (224 B/row instead of 440).  Afterwards (k_vastro, k_vshared) v' = z/beta - beta v, which is
+// algebraically the P&S step b (u = u_hat/beta).  Astro z goes to zA (scatter-free, per star), the shared slice to
+// z_sh exactly as in aprod2.  The ring is shallower (8-row stages) because v_instr (gathers) and z_instr
+// (accumulator) both live in shared memory.
+constexpr int kFRows = 8, kFStages = 4;
+using FRing = RingT<kFRows, kFStages>;
+constexpr int kSmemMaxBytes = 232448;  // 227 KB opt-in per CTA on sm_100
+constexpr int kFusedInstrMax = (kSmemMaxBytes - FRing::kBytes - FRing::kBars) / 16;
+
+template <bool SMEM_INSTR>
+__global__ void __launch_bounds__(kThreads, 1)
+    k_fused(SysView S, const double* __restrict__ x, double* __restrict__ u, double* __restrict__ zA,
+            double* __restrict__ zsh, double* __restrict__ part, double* __restrict__ cpart,
+            const DevState* __restrict__ st) {
+  extern __shared__ __align__(128) unsigned char dsm[];
+  if (st->halted) return;
+  double* sh_x = reinterpret_cast<double*>(dsm + FRing::kBytes + FRing::kBars);
+  double* sh_z = sh_x + S.n_instr;
+  if (SMEM_INSTR) {
+    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
+      sh_x[i] = x[S.I0 + i];
+      sh_z[i] = 0.0;
+    }
+    __syncthreads();
+  }
+  const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2, wid = threadIdx.x >> 5;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const double uscale = st->u_scale;
+  const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
+  FRing R;
+  R.setup(S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
+  R.prologue(lane);
+  const double* xatt0 = x + S.A0 + j;
+  const double* xatt1 = xatt0 + S.n_axis;
+  const double* xatt2 = xatt1 + S.n_axis;
+  const double* xins = SMEM_INSTR ? sh_x : x + S.I0;
+  const double vglob = S.n_glob ? __ldg(x + S.G0) : 0.0;
+  double* zatt0 = zsh + j;
+  double* zatt1 = zatt0 + S.n_axis;
+  double* zatt2 = zatt1 + S.n_axis;
+  double* z_ins = SMEM_INSTR ? sh_z : zsh + S.n_att;
+  int64_t s = s_lo, bound = S.star_ptr[s_lo + 1];
+  AstroCache ac;
+  ac.init(x, s_lo, s_hi, j);
+  int64_t cs = s_lo;
+  int64_t cs_end = (cs < s_hi) ? S.star_ptr[cs + 1] : 0;
+  double b2 = 0.0, gacc = 0.0, acc0 = 0.0, acc1 = 0.0;
+
+  auto finalize = [&](int64_t star) {  // z of the star's 5 astro columns -> zA (no atomics)
+    double z0 = acc0, z1 = acc1;
+    z0 += __shfl_xor_sync(0xffffffffu, z0, 4);
+    z0 += __shfl_xor_sync(0xffffffffu, z0, 8);
+    z0 += __shfl_xor_sync(0xffffffffu, z0, 16);
+    z1 += __shfl_xor_sync(0xffffffffu, z1, 4);
+    z1 += __shfl_xor_sync(0xffffffffu, z1, 8);
+    z1 += __shfl_xor_sync(0xffffffffu, z1, 16);
+    if (lane < 4) {
+      zA[5 * star + j] = z0;
+      if (j == 0) zA[5 * star + 4] = z1;
+    }
+  };
+
+  double* up = u + R.r_lo + r;
+  double unext = (R.r_lo + r < R.r_hi) ? __ldg(up) : 0.0;
+  int64_t row0 = R.r_lo;
+  for (int64_t k = 0; k < R.nst; ++k, row0 += kFRows, up += kFRows) {
+    const double uold = unext;
+    unext = (row0 + kFRows + r < R.r_hi) ? __ldg(up + kFRows) : 0.0;
+    const unsigned char* stg = R.wait();
+    const int64_t row = row0 + r;
+    const bool valid = row < R.r_hi;
+    double v[6];
+    IdxRec rec;
+    stage_row<kFRows>(stg, r, j, v, rec);
+    if (valid && track_star(S, row, s, bound)) ac.move_to(x, s, s_hi, j);
+    const int k0 = valid ? rec.k0 : 0;
+    const uint32_t i4 = valid ? ic4_of(rec, j) : 0u, i5 = valid ? ic5_of(rec, j) : 0u;
+    const double g1 = __ldg(xatt0 + k0), g2 = __ldg(xatt1 + k0), g3 = __ldg(xatt2 + k0);
+    const double g4 = SMEM_INSTR ? xins[i4] : __ldg(xins + i4);
+    const double gi5 = SMEM_INSTR ? xins[i5] : __ldg(xins + i5);
+    const double g5 = j == 0 ? ac.c4 : (j == 3 ? vglob : gi5);
+    double p = v[0] * ac.cj;
+    p = fma(v[1], g1, p);
+    p = fma(v[2], g2, p);
+    p = fma(v[3], g3, p);
+    p = fma(v[4], g4, p);
+    p = fma(v[5], g5, p);
+    p += __shfl_xor_sync(0xffffffffu, p, 1);
+    p += __shfl_xor_sync(0xffffffffu, p, 2);
+    const double un = valid ? p - uscale * uold : 0.0;  // identical in the row's 4 lanes
+    if (valid && j == 0) {
+      up[0] = un;
+      b2 = fma(un, un, b2);
+    }
+    double c[6];
+#pragma unroll
+    for (int t = 0; t < 6; ++t) c[t] = v[t] * un;
+    double* ia[2] = {z_ins, z_ins};
+    double iv[2] = {0.0, 0.0};
+    bool ion[2] = {false, false};
+    if (valid) {
+      atomicAdd(zatt0 + k0, c[1]);
+      atomicAdd(zatt1 + k0, c[2]);
+      atomicAdd(zatt2 + k0, c[3]);
+      if (SMEM_INSTR) {
+        ia[0] = z_ins + i4; iv[0] = c[4]; ion[0] = true;
+        ia[1] = z_ins + i5; iv[1] = c[5]; ion[1] = (j == 1 || j == 2);
+      } else {
+        atomicAdd(z_ins + i4, c[4]);
+        if (j == 1 || j == 2) atomicAdd(z_ins + i5, c[5]);
+      }
+      if (j == 3) gacc += c[5];
+    }
+    // astrometric: segmented by star
+    const double c0 = c[0], c5 = (j == 0) ? c[5] : 0.0;
+    {
+      const int64_t step_end = row0 + 8 < R.r_hi ? row0 + 8 : R.r_hi;
+      while (true) {
+        if (valid && s == cs) { acc0 += c0; acc1 += c5; }
+        if (cs < s_hi && cs_end <= step_end) {
+          finalize(cs);
+          acc0 = 0.0; acc1 = 0.0;
+          ++cs;
+          if (cs >= s_hi) break;
+          cs_end = S.star_ptr[cs + 1];
+        } else {
+          break;
+        }
+      }
+    }
+    if (SMEM_INSTR) smem_add_n<2>(ia, iv, ion);
+    R.release(lane);
+  }
+  while (cs < s_hi) {
+    acc0 = 0.0; acc1 = 0.0;
+    finalize(cs);
+    ++cs;
+  }
+  if (S.n_glob) {
+    gacc = warp_sum(gacc);
+    if (lane == 0 && gacc != 0.0) atomicAdd(zsh + S.n_att + S.n_instr, gacc);
+  }
+  b2 = warp_sum(b2);
+  if (lane == 0) part[gw] = b2;
+  for (int64_t c = gw; c < S.n_chunks; c += W) {  // constraint rows: owned-entry partial dots with v
+    double acc = 0.0;
+    for (int64_t e = S.ch_beg[c] + lane; e < S.ch_end[c]; e += 32) acc = fma(S.cval[e], __ldg(x + S.ccol[e]), acc);
+    acc = warp_sum(acc);
+    if (lane == 0) cpart[c] = acc;
+  }
+  if (SMEM_INSTR) {
+    __syncthreads();
+    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
+      const double vv = sh_z[i];
+      if (vv != 0.0) atomicAdd(zsh + S.n_att + i, vv);
+    }
+  }
+}
+
+// Fused mode, after k_beta: astro columns v' = (zA + constraint entries . u_hat_c) / beta - beta v  (P&S step b),
+// per-block alpha^2 partials; shared-column constraint entries added to z_sh (rank 0) before AR2 / k_vshared.
+__global__ void __launch_bounds__(kRedThreads)
+    k_vastro(SysView S, double* __restrict__ v, const double* __restrict__ zA, const double* __restrict__ uc,
+             double* __restrict__ zsh, double* __restrict__ part, const DevState* __restrict__ st,
+             int do_shared_constr) {
+  if (st->halted || !st->beta_pos) return;
+  const double ib = st->inv_beta, beta = st->beta;
+  const int64_t na = 5 * S.n_stars;
+  double a2 = 0.0;
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < na; c += (int64_t)gridDim.x * blockDim.x) {
+    double z = zA[c];
+    const int64_t star = c / 5;
+    if (star < S.n_cs) {
+      const int a = (int)(c - 5 * star);
+      for (int64_t e = S.cs_ptr[star]; e < S.cs_ptr[star + 1]; ++e) {
+        const int ak = S.cs_ak[e];
+        if ((ak & 0xff) == a) z += S.cval[S.cs_e[e]] * uc[ak >> 8];
+      }
+    }
+    const double vn = z * ib - beta * v[c];
+    v[c] = vn;
+    a2 = fma(vn, vn, a2);
+  }
+  a2 = block_sum<kRedThreads>(a2);
+  if (threadIdx.x == 0) part[blockIdx.x] = a2;
+  if (do_shared_constr)
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < S.n_csh;
+         e += (int64_t)gridDim.x * blockDim.x)
+      atomicAdd(zsh + S.csh_idx[e], S.cval[S.csh_e[e]] * uc[S.csh_k[e]]);
 }
 
 // ------------------------------------------------------------------------------------------------ scale rows (O-PREC)
@@ -661,12 +923,12 @@ __global__ void k_cdot_add(SysView S, const double* __restrict__ cpart, const do
 
 __global__ void __launch_bounds__(kRedThreads)
     k_vshared(int64_t n_sh, double* __restrict__ vsh, double* __restrict__ zsh, double* __restrict__ part,
-              const DevState* __restrict__ st) {
+              const DevState* __restrict__ st, int fused) {
   if (st->halted || !st->beta_pos) return;
-  const double beta = st->beta;
+  const double beta = st->beta, zs = fused ? st->inv_beta : 1.0;  // fused mode: z = A^T u_hat (unnormalised)
   double a2 = 0.0;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_sh; i += (int64_t)gridDim.x * blockDim.x) {
-    const double vn = zsh[i] - beta * vsh[i];
+    const double vn = zsh[i] * zs - beta * vsh[i];
     vsh[i] = vn;
     zsh[i] = 0.0;
     a2 = fma(vn, vn, a2);
@@ -954,10 +1216,36 @@ cudaError_t launch_cdot_add(const SysView& S, const double* cpart, const double*
   return cudaGetLastError();
 }
 cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* part, int nblk, const DevState* st,
-                           cudaStream_t s) {
-  k_vshared<<<nblk, kRedThreads, 0, s>>>(S.n_sh, vsh, zsh, part, st);
+                           int fused, cudaStream_t s) {
+  k_vshared<<<nblk, kRedThreads, 0, s>>>(S.n_sh, vsh, zsh, part, st, fused);
   return cudaGetLastError();
 }
+template <bool SM>
+static cudaError_t fz(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh, double* part,
+                      double* cpart, const DevState* st, cudaStream_t s) {
+  const size_t smem = FRing::kBytes + FRing::kBars + (SM ? 2 * (size_t)S.n_instr * sizeof(double) : 0);
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(k_fused<SM>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemMaxBytes);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  k_fused<SM><<<grid, kThreads, smem, s>>>(S, x, u, zA, zsh, part, cpart, st);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh,
+                         double* part, double* cpart, const DevState* st, cudaStream_t s) {
+  return S.n_instr <= kFusedInstrMax ? fz<true>(S, grid, x, u, zA, zsh, part, cpart, st, s)
+                                     : fz<false>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+}
+
+cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const double* uc, double* zsh, double* part,
+                          int nblk, const DevState* st, int do_shared_constr, cudaStream_t s) {
+  k_vastro<<<nblk, kRedThreads, 0, s>>>(S, v, zA, uc, zsh, part, st, do_shared_constr);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_add_shared(double* xsh, double* zsh, int64_t n, int mode, cudaStream_t s) {
   k_add_shared<<<vec_grid(n, 148 * 4), kRedThreads, 0, s>>>(xsh, zsh, n, mode);
   return cudaGetLastError();

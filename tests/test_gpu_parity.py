@@ -173,7 +173,7 @@ def reversed_control(S):
     return C2
 
 
-def free_run_curves(avu, w, kmax=30):
+def free_run_curves(avu, w, kmax=30, fused=False):
     s = gpu_solver(avu, w)
     s.precondition()
     S = oracle.System(w)
@@ -184,7 +184,7 @@ def free_run_curves(avu, w, kmax=30):
     _, hc = oracle_trace(Cs, kmax, atol=0, btol=0, conlim=0)
     n = S.n_rows
     ctrl, gpu = [], []
-    s.init(itn_limit=100, atol=0, btol=0, conlim=0, fixed_count=True)
+    s.init(itn_limit=100, atol=0, btol=0, conlim=0, fixed_count=True, fused=fused)
     for k in range(1, kmax + 1):
         s.iterate(1)
         st, vec = s.get_state()
@@ -196,9 +196,10 @@ def free_run_curves(avu, w, kmax=30):
     return s, S, res_o, np.array(ctrl), np.array(gpu)
 
 
+@pytest.mark.parametrize("fused", [False, True], ids=["twopass", "fused"])
 @pytest.mark.parametrize("w", [W.C1, W.C1C], ids=["C1", "C1c"])
-def test_lsqr_free_run_and_converged(avu, w):
-    s, S, res_o, ctrl, gpu = free_run_curves(avu, w)
+def test_lsqr_free_run_and_converged(avu, w, fused):
+    s, S, res_o, ctrl, gpu = free_run_curves(avu, w, fused=fused)
     print("\nfree-run rel diff per iteration (control = oracle with reordered sums | GPU):")
     for k, (c, g) in enumerate(zip(ctrl, gpu), 1):
         print(f"  k={k:2d}  control {c:.2e}  gpu {g:.2e}")
@@ -226,15 +227,16 @@ def test_lsqr_free_run_and_converged(avu, w):
     s.close()
 
 
+@pytest.mark.parametrize("fused", [False, True], ids=["twopass", "fused"])
 @pytest.mark.parametrize("w", [W.C1, W.C1C], ids=["C1", "C1c"])
-def test_lsqr_teacher_forced_step(avu, w):
+def test_lsqr_teacher_forced_step(avu, w, fused):
     s = gpu_solver(avu, w)
     s.precondition()
     S = oracle.System(w)
     S.apply_precond()
     S.vals[:] = s.get_system(with_b=False)["vals"]
     _, hist = oracle_trace(S, 60, atol=0, btol=0, conlim=0)
-    s.init(itn_limit=1000, atol=0, btol=0, conlim=0, fixed_count=True)
+    s.init(itn_limit=1000, atol=0, btol=0, conlim=0, fixed_count=True, fused=fused)
     for k in (1, 2, 5, 13, 30, 59):
         so, u, v, w_, x, var = hist[k - 1]
         sc = dict(so); sc["itn"] = k; sc["istop"] = 0; sc["istop_first"] = 0; sc["halted"] = 0
@@ -304,14 +306,32 @@ def test_lsqr_damped(avu):
     s.close()
 
 
-def test_graph_and_eager_agree(avu):
+def test_graph_eager_fused_agree(avu):
     w = W.C1C
     outs = []
-    for g in (True, False):
+    for g, f in ((True, False), (False, False), (True, True), (False, True)):
         s = gpu_solver(avu, w)
         s.precondition()
-        outs.append(s.solve(itn_limit=100, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=g))
+        outs.append(s.solve(itn_limit=160, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=g, fused=f))
         s.close()
     # x agrees once converged (before convergence two valid FP64 runs differ, SURVEY EXP-3/4)
-    assert outs[0]["itn"] == outs[1]["itn"] == 100
-    assert rel(outs[0]["x"], outs[1]["x"]) <= 1e-9
+    for o in outs[1:]:
+        assert o["itn"] == 160
+        assert rel(o["x"], outs[0]["x"]) <= 1e-9
+
+
+@pytest.mark.parametrize("fused", [False, True], ids=["twopass", "fused"])
+def test_lsqr_C2_full_vs_oracle(avu, fused):
+    """configs[1] at full size (5 M rows, constraints, preconditioned): 100 fixed iterations vs the oracle."""
+    w = W.C2
+    s = gpu_solver(avu, w)
+    s.precondition()
+    out = s.solve(itn_limit=100, atol=0, btol=0, conlim=0, fixed_count=True, fused=fused)
+    S = oracle.System(w)
+    ro = oracle.solve_system(S, itn_limit=100, atol=0, btol=0, conlim=0, fixed_count=True)
+    print(f"C2 fused={fused}: x rel diff {rel(out['x'], ro['x']):.2e}, r1norm {out['r1norm']:.10e} vs "
+          f"{ro['r1norm']:.10e}, arnorm {out['arnorm']:.3e} vs {ro['arnorm']:.3e}")
+    assert out["itn"] == 100
+    assert abs(out["r1norm"] - ro["r1norm"]) <= 1e-10 * ro["r1norm"]
+    assert rel(out["x"], ro["x"]) <= 1e-9
+    s.close()

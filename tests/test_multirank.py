@@ -100,7 +100,7 @@ def test_gloo_two_rank_decomposition_cpu():
 
 
 # ------------------------------------------------------------------------------------------------ GPU
-def _gpu_worker(rank, world, port, q, itn):
+def _gpu_worker(rank, world, port, q, itn, fused):
     try:
         import sys
         sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -112,7 +112,7 @@ def _gpu_worker(rank, world, port, q, itn):
         s = avu.Solver.synthetic(w, rank=rank, nranks=world, comm="callback")
         s.precondition()
         D = s.get_precond()
-        out = s.solve(itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=False)
+        out = s.solve(itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=False, fused=fused)
         # plain products through the ABI
         xg = torch.ones(s.n_local_cols, dtype=torch.float64, device="cuda")
         yg = torch.zeros(s.n_local_rows + s.n_constr, dtype=torch.float64, device="cuda")
@@ -130,14 +130,15 @@ def _gpu_worker(rank, world, port, q, itn):
 
 
 @pytest.mark.gpu
-def test_gpu_two_rank_lsqr_matches_single_rank(cuda_device):
+@pytest.mark.parametrize("fused", [False, True], ids=["twopass", "fused"])
+def test_gpu_two_rank_lsqr_matches_single_rank(cuda_device, fused):
     import torch
     import paper_conf_sc_malenzacsbvba24_b200 as avu
     itn = 160  # converged (x parity needs convergence, SURVEY EXP-3)
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    ps = [ctx.Process(target=_gpu_worker, args=(r, 2, port, q, itn)) for r in range(2)]
+    ps = [ctx.Process(target=_gpu_worker, args=(r, 2, port, q, itn, fused)) for r in range(2)]
     for p in ps:
         p.start()
     outs = [q.get(timeout=600) for _ in range(2)]
