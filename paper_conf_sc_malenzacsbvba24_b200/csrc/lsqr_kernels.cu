@@ -6,6 +6,8 @@
 // t=5 {astro 4, instr 4, instr 5, global}[j].  Each of the 6 loads of a warp instruction reads 8 rows x 32
 // contiguous bytes, so every fetched byte of A is used; the 4 lanes of a row hit 4 consecutive attitude columns,
 // which makes the attitude gathers (aprod1) and REDs (aprod2) sector-coalesced.
+#include <type_traits>
+
 #include "lsqr_internal.cuh"
 
 namespace lsqr {
@@ -611,7 +613,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 constexpr int kFRows = 8, kFStages = 4;
 using FRing = RingT<kFRows, kFStages>;
 constexpr int kSmemMaxBytes = 232448;  // 227 KB opt-in per CTA on sm_100
-constexpr int kFusedInstrMax = (kSmemMaxBytes - FRing::kBytes - FRing::kBars) / 16;
+constexpr int kFusedInstrMax = (kSmemMaxBytes - FRing::kBytes - FRing::kBars) / 16 - 2;
 
 template <bool SMEM_INSTR>
 __global__ void __launch_bounds__(kThreads, 1)
@@ -620,13 +622,15 @@ __global__ void __launch_bounds__(kThreads, 1)
             const DevState* __restrict__ st) {
   extern __shared__ __align__(128) unsigned char dsm[];
   if (st->halted) return;
+  // shared memory: [ring | mbarriers | v_instr (n_instr) + v_glob | z_instr accumulator (n_instr)]
   double* sh_x = reinterpret_cast<double*>(dsm + FRing::kBytes + FRing::kBars);
-  double* sh_z = sh_x + S.n_instr;
+  double* sh_z = sh_x + S.n_instr + 2;
   if (SMEM_INSTR) {
     for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
       sh_x[i] = x[S.I0 + i];
       sh_z[i] = 0.0;
     }
+    if (threadIdx.x == 0) sh_x[S.n_instr] = S.n_glob ? x[S.G0] : 0.0;
     __syncthreads();
   }
   const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2, wid = threadIdx.x >> 5;
@@ -634,26 +638,35 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const double uscale = st->u_scale;
   const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
+  const int64_t r_lo = S.star_ptr[s_lo];
+  const int nrows = (int)(S.star_ptr[s_hi] - r_lo);  // rows of this warp (< 2^31)
   FRing R;
-  R.setup(S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
+  R.setup(S, dsm, wid, lane, r_lo, r_lo + nrows);
   R.prologue(lane);
+  // per-lane loop invariants
   const double* xatt0 = x + S.A0 + j;
   const double* xatt1 = xatt0 + S.n_axis;
   const double* xatt2 = xatt1 + S.n_axis;
-  const double* xins = SMEM_INSTR ? sh_x : x + S.I0;
-  const double vglob = S.n_glob ? __ldg(x + S.G0) : 0.0;
   double* zatt0 = zsh + j;
   double* zatt1 = zatt0 + S.n_axis;
   double* zatt2 = zatt1 + S.n_axis;
-  double* z_ins = SMEM_INSTR ? sh_z : zsh + S.n_att;
-  int64_t s = s_lo, bound = S.star_ptr[s_lo + 1];
-  AstroCache ac;
-  ac.init(x, s_lo, s_hi, j);
+  const double* xins_g = x + S.I0;      // (non-smem fallback)
+  double* zins_g = zsh + S.n_att;
+  const double vglob_g = S.n_glob ? __ldg(x + S.G0) : 0.0;
+  const double m0 = (j == 0) ? 1.0 : 0.0;                 // lane 0 of a row holds astro slot 4 at t=5
+  const double m3 = (j == 3 && S.n_glob) ? 1.0 : 0.0;     // lane 3 holds the global slot at t=5
+  const bool t5_ins = (j == 1 || j == 2);                 // lanes 1, 2 hold instr 4, 5 at t=5
+  double* const urow = u + r_lo + r;
+
+  // warp-uniform star state: cs = star of the next row to process; its astro values (cj, c4) and the next star's
   int64_t cs = s_lo;
-  int64_t cs_end = (cs < s_hi) ? S.star_ptr[cs + 1] : 0;
+  int cs_end = (cs < s_hi) ? (int)(S.star_ptr[cs + 1] - r_lo) : nrows;
+  double cj = 0.0, c4 = 0.0, nj = 0.0, n4 = 0.0;
+  if (cs < s_hi) { cj = __ldg(x + 5 * cs + j); c4 = __ldg(x + 5 * cs + 4); }
+  if (cs + 1 < s_hi) { nj = __ldg(x + 5 * (cs + 1) + j); n4 = __ldg(x + 5 * (cs + 1) + 4); }
   double b2 = 0.0, gacc = 0.0, acc0 = 0.0, acc1 = 0.0;
 
-  auto finalize = [&](int64_t star) {  // z of the star's 5 astro columns -> zA (no atomics)
+  auto advance = [&]() {  // star cs is complete: its 5 astro sums -> zA (scatter-free), move to cs+1
     double z0 = acc0, z1 = acc1;
     z0 += __shfl_xor_sync(0xffffffffu, z0, 4);
     z0 += __shfl_xor_sync(0xffffffffu, z0, 8);
@@ -662,87 +675,119 @@ __global__ void __launch_bounds__(kThreads, 1)
     z1 += __shfl_xor_sync(0xffffffffu, z1, 8);
     z1 += __shfl_xor_sync(0xffffffffu, z1, 16);
     if (lane < 4) {
-      zA[5 * star + j] = z0;
-      if (j == 0) zA[5 * star + 4] = z1;
+      zA[5 * cs + j] = z0;
+      if (j == 0) zA[5 * cs + 4] = z1;
     }
+    acc0 = 0.0;
+    acc1 = 0.0;
+    ++cs;
+    cs_end = (cs < s_hi) ? (int)(S.star_ptr[cs + 1] - r_lo) : nrows;
+    cj = nj;
+    c4 = n4;
+    if (cs + 1 < s_hi) { nj = __ldg(x + 5 * (cs + 1) + j); n4 = __ldg(x + 5 * (cs + 1) + 4); }
   };
+  while (cs < s_hi && cs_end <= 0) advance();  // leading empty stars
 
-  double* up = u + R.r_lo + r;
-  double unext = (R.r_lo + r < R.r_hi) ? __ldg(up) : 0.0;
-  int64_t row0 = R.r_lo;
-  for (int64_t k = 0; k < R.nst; ++k, row0 += kFRows, up += kFRows) {
-    const double uold = unext;
-    unext = (row0 + kFRows + r < R.r_hi) ? __ldg(up + kFRows) : 0.0;
-    const unsigned char* stg = R.wait();
-    const int64_t row = row0 + r;
-    const bool valid = row < R.r_hi;
+  // one 8-row group: gathers, row dot, u_hat update, contributions.  CHECK: tail / star-boundary path with
+  // per-lane validity and per-lane star; otherwise every lane's row is valid and in star cs.
+  auto group = [&](const unsigned char* stg, int g0, double uold, auto check_tag) {
+    constexpr bool CHECK = decltype(check_tag)::value;
+    const int rel = g0 + r;
+    const bool valid = !CHECK || rel < nrows;
     double v[6];
     IdxRec rec;
     stage_row<kFRows>(stg, r, j, v, rec);
-    if (valid && track_star(S, row, s, bound)) ac.move_to(x, s, s_hi, j);
-    const int k0 = valid ? rec.k0 : 0;
-    const uint32_t i4 = valid ? ic4_of(rec, j) : 0u, i5 = valid ? ic5_of(rec, j) : 0u;
+    double xj = cj, x4 = c4;
+    int64_t my_s = cs;
+    if (CHECK) {
+      if (valid) {
+        int my_end = cs_end;
+        while (my_end <= rel) {
+          ++my_s;
+          my_end = (int)(S.star_ptr[my_s + 1] - r_lo);
+        }
+        if (my_s == cs + 1) { xj = nj; x4 = n4; }
+        else if (my_s != cs) { xj = __ldg(x + 5 * my_s + j); x4 = __ldg(x + 5 * my_s + 4); }
+      } else {
+        rec.k0 = 0; rec.ic01 = rec.ic23 = rec.ic45 = 0;
+#pragma unroll
+        for (int t = 0; t < 6; ++t) v[t] = 0.0;
+      }
+    }
+    const int k0 = rec.k0;
+    const uint32_t i4 = ic4_of(rec, j);
+    const uint32_t i5 = (j == 3) ? (uint32_t)S.n_instr : ic5_of(rec, j);
     const double g1 = __ldg(xatt0 + k0), g2 = __ldg(xatt1 + k0), g3 = __ldg(xatt2 + k0);
-    const double g4 = SMEM_INSTR ? xins[i4] : __ldg(xins + i4);
-    const double gi5 = SMEM_INSTR ? xins[i5] : __ldg(xins + i5);
-    const double g5 = j == 0 ? ac.c4 : (j == 3 ? vglob : gi5);
-    double p = v[0] * ac.cj;
-    p = fma(v[1], g1, p);
+    double g4, g5;
+    if (SMEM_INSTR) {
+      g4 = sh_x[i4];
+      g5 = sh_x[i5];
+    } else {
+      g4 = __ldg(xins_g + i4);
+      g5 = (j == 3) ? vglob_g : __ldg(xins_g + ic5_of(rec, j));
+    }
+    g5 = (j == 0) ? x4 : g5;
+    double p = fma(v[1], g1, v[0] * xj);  // two short chains instead of one long one
+    double p2 = fma(v[4], g4, v[3] * g3);
     p = fma(v[2], g2, p);
-    p = fma(v[3], g3, p);
-    p = fma(v[4], g4, p);
-    p = fma(v[5], g5, p);
+    p2 = fma(v[5], g5, p2);
+    p += p2;
     p += __shfl_xor_sync(0xffffffffu, p, 1);
     p += __shfl_xor_sync(0xffffffffu, p, 2);
     const double un = valid ? p - uscale * uold : 0.0;  // identical in the row's 4 lanes
-    if (valid && j == 0) {
-      up[0] = un;
+    if (j == 0 && valid) {
+      urow[g0] = un;
       b2 = fma(un, un, b2);
     }
-    double c[6];
-#pragma unroll
-    for (int t = 0; t < 6; ++t) c[t] = v[t] * un;
-    double* ia[2] = {z_ins, z_ins};
-    double iv[2] = {0.0, 0.0};
-    bool ion[2] = {false, false};
+    const double c1 = v[1] * un, c2 = v[2] * un, c3 = v[3] * un, c4v = v[4] * un, c5 = v[5] * un;
     if (valid) {
-      atomicAdd(zatt0 + k0, c[1]);
-      atomicAdd(zatt1 + k0, c[2]);
-      atomicAdd(zatt2 + k0, c[3]);
-      if (SMEM_INSTR) {
-        ia[0] = z_ins + i4; iv[0] = c[4]; ion[0] = true;
-        ia[1] = z_ins + i5; iv[1] = c[5]; ion[1] = (j == 1 || j == 2);
-      } else {
-        atomicAdd(z_ins + i4, c[4]);
-        if (j == 1 || j == 2) atomicAdd(z_ins + i5, c[5]);
-      }
-      if (j == 3) gacc += c[5];
+      atomicAdd(zatt0 + k0, c1);
+      atomicAdd(zatt1 + k0, c2);
+      atomicAdd(zatt2 + k0, c3);
     }
-    // astrometric: segmented by star
-    const double c0 = c[0], c5 = (j == 0) ? c[5] : 0.0;
-    {
-      const int64_t step_end = row0 + 8 < R.r_hi ? row0 + 8 : R.r_hi;
+    if (SMEM_INSTR) {
+      double* ia[2] = {sh_z + i4, sh_z + i5};
+      const double iv[2] = {c4v, c5};
+      const bool ion[2] = {valid, valid && t5_ins};
+      smem_add_n<2>(ia, iv, ion);
+    } else if (valid) {
+      atomicAdd(zins_g + i4, c4v);
+      if (t5_ins) atomicAdd(zins_g + ic5_of(rec, j), c5);
+    }
+    gacc = fma(c5, m3, gacc);
+    const double c0 = v[0] * un, c5a = c5 * m0;
+    if (!CHECK) {
+      acc0 += c0;
+      acc1 += c5a;
+    } else {  // segmented by star inside the group
+      const int g1end = g0 + 8 < nrows ? g0 + 8 : nrows;
       while (true) {
-        if (valid && s == cs) { acc0 += c0; acc1 += c5; }
-        if (cs < s_hi && cs_end <= step_end) {
-          finalize(cs);
-          acc0 = 0.0; acc1 = 0.0;
-          ++cs;
-          if (cs >= s_hi) break;
-          cs_end = S.star_ptr[cs + 1];
-        } else {
-          break;
-        }
+        if (valid && my_s == cs) { acc0 += c0; acc1 += c5a; }
+        if (cs < s_hi && cs_end <= g1end) advance();
+        else break;
       }
     }
-    if (SMEM_INSTR) smem_add_n<2>(ia, iv, ion);
+  };
+
+  const int nst = (nrows + kFRows - 1) / kFRows;
+  double uq0 = (r < nrows) ? __ldg(urow) : 0.0;            // u_hat of stage k (register queue, 2 deep)
+  double uq1 = (kFRows + r < nrows) ? __ldg(urow + kFRows) : 0.0;
+  for (int k = 0; k < nst; ++k) {
+    const int g0 = k * kFRows;
+    const double uold = uq0;
+    uq0 = uq1;
+    uq1 = (g0 + 2 * kFRows + r < nrows) ? __ldg(urow + g0 + 2 * kFRows) : 0.0;
+    const unsigned char* stg = R.wait();
+    const bool fast = (g0 + kFRows <= nrows) && (cs_end >= g0 + kFRows);
+    if (fast) {
+      group(stg, g0, uold, std::false_type{});
+      while (cs < s_hi && cs_end <= g0 + kFRows) advance();
+    } else {
+      group(stg, g0, uold, std::true_type{});
+    }
     R.release(lane);
   }
-  while (cs < s_hi) {
-    acc0 = 0.0; acc1 = 0.0;
-    finalize(cs);
-    ++cs;
-  }
+  while (cs < s_hi) advance();  // empty trailing stars
   if (S.n_glob) {
     gacc = warp_sum(gacc);
     if (lane == 0 && gacc != 0.0) atomicAdd(zsh + S.n_att + S.n_instr, gacc);
@@ -1223,7 +1268,7 @@ cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* p
 template <bool SM>
 static cudaError_t fz(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh, double* part,
                       double* cpart, const DevState* st, cudaStream_t s) {
-  const size_t smem = FRing::kBytes + FRing::kBars + (SM ? 2 * (size_t)S.n_instr * sizeof(double) : 0);
+  const size_t smem = FRing::kBytes + FRing::kBars + (SM ? (2 * (size_t)S.n_instr + 2) * sizeof(double) : 0);
   static bool attr_set = false;
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(k_fused<SM>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemMaxBytes);
