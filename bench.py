@@ -6,7 +6,9 @@
     torchrun --nproc-per-node N bench.py --gpus N ...                     # multi-GPU, weak scaling
 
 A "step" is one LSQR iteration (aprod1 + beta + aprod2 + shared-slice update + scalar recurrence + column update,
-SURVEY §8(a) a3-a9) over the whole synthetic system; in fixed-count mode as in the paper.  Weak
+SURVEY §8(a) a3-a9) over the whole synthetic system; in fixed-count mode as in the paper.  Default
+variant: the fused single pass (SURVEY §8(f) NEXT-1, A read once per iteration); `--two-pass` times aprod1 and
+aprod2 as separate passes.  Weak
 scaling: every GPU holds one copy of the configuration's shape (n_stars, n_obs multiplied by N).  Inputs (A: 1 GB
 at C2) are larger than L2 (126 MB), so no L2 flush is needed between iterations.
 """
@@ -107,12 +109,13 @@ def algorithmic_bytes(w, n_rows, n_stars, n_sh, n_cols):
     return ap1, ap2, it
 
 
-def load_traffic(kernel):
+def load_traffic(workload, kernel):
+    """DRAM bytes per launch of `kernel` from a committed ncu --set full capture of the same workload, or None."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(p):
         with open(p) as f:
             d = json.load(f)
-        return d.get(kernel)
+        return d.get(workload, {}).get(kernel)
     return None
 
 
@@ -295,7 +298,7 @@ def run_ours(args):
         "config": config_block(w, n, args, {"total_rows": w.n_obs, "setup_s": round(t_setup, 3)}),
         "roofline": {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak,
                      "peak_kind": f"{peak_kind} (MEASURED_PEAKS.json hbm_gbs, copy; burst)", "unit": "GB/s",
-                     "frac": round(achieved / peak, 4), "traffic": load_traffic(kname),
+                     "frac": round(achieved / peak, 4), "traffic": load_traffic(w.name if n == 1 else None, kname),
                      "algorithmic_bytes_per_launch": kb, "avg_launch_ms": round(kms, 4)},
         "iteration_roofline": {"algorithmic_bytes": it_b, "achieved_GBps": round(it_b / (ms_step * 1e-3) / 1e9, 1),
                                "frac": round(it_b / (ms_step * 1e-3) / 1e9 / peak, 4),
@@ -331,7 +334,9 @@ def main():
     ap.add_argument("--no-e2e", dest="e2e", action="store_false")
     ap.add_argument("--no-cpu-baseline", dest="cpu_baseline", action="store_false")
     ap.add_argument("--cpu-iters", type=int, default=3)
-    ap.add_argument("--fused", action="store_true", help="fused single-pass iteration (SURVEY 8(f) NEXT-1)")
+    ap.add_argument("--fused", dest="fused", action="store_true", default=True,
+                    help="fused single-pass iteration (SURVEY 8(f) NEXT-1; default)")
+    ap.add_argument("--two-pass", dest="fused", action="store_false", help="two-pass iteration (aprod1 then aprod2)")
     args = ap.parse_args()
     if args.warmup < 3:
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)

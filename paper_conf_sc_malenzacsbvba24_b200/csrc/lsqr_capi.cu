@@ -93,7 +93,8 @@ struct lsqr_ctx {
   std::vector<void*> allocs;
   double *vals = nullptr, *u = nullptr, *v = nullptr, *w = nullptr, *x = nullptr, *var = nullptr, *D = nullptr;
   double *zsh = nullptr, *part_rows = nullptr, *part_a2 = nullptr, *cpart = nullptr, *part_sh = nullptr;
-  double *zA = nullptr, *part_va = nullptr;  // fused mode: astro z (A^T u_hat) and alpha^2 partials of k_vastro
+  double *zA = nullptr, *part_va = nullptr;
+  double* ingest = nullptr;  // lsqr_set_system staging (lazily allocated)  // fused mode: astro z (A^T u_hat) and alpha^2 partials of k_vastro
   double *part_wa = nullptr, *part_ws = nullptr, *part_g1 = nullptr, *ar1 = nullptr, *uc = nullptr,
          *ucn = nullptr, *crhs = nullptr, *tmp = nullptr, *tmax = nullptr;
   IdxRec* idx = nullptr;
@@ -500,13 +501,13 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   std::vector<int32_t> ch_row;
   std::vector<int64_t> ch_beg, ch_end;
   std::vector<int64_t> cs_ptr;
-  std::vector<int32_t> cs_ak;
+  std::vector<int32_t> cs_k;
   std::vector<int64_t> cs_e, csh_idx, csh_e;
   std::vector<int32_t> csh_k;
   std::vector<double> crhs(std::max<int64_t>(nc, 1), 0.0);
   if (nc > 0) {
     const int64_t A0l = 5 * h->n_loc_stars;
-    std::vector<std::vector<std::pair<int32_t, int64_t>>> by_star;  // local star -> (ak, entry)
+    std::vector<std::vector<std::pair<int32_t, int64_t>>> by_col;  // local astro column -> (row k, entry)
     for (int64_t k = 0; k < nc; ++k) {
       if (cons->rhs) crhs[k] = cons->rhs[k];
       const int64_t row_first = (int64_t)cval.size();
@@ -516,9 +517,8 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
         if (c < A0g) {
           if (c < 5 * h->star_begin || c >= 5 * h->star_end) continue;
           lc = c - 5 * h->star_begin;
-          const int64_t sl = lc / 5;
-          if ((int64_t)by_star.size() <= sl) by_star.resize(sl + 1);
-          by_star[sl].push_back({(int32_t)((lc % 5) | (k << 8)), (int64_t)cval.size()});
+          if ((int64_t)by_col.size() <= lc) by_col.resize(lc + 1);
+          by_col[lc].push_back({(int32_t)k, (int64_t)cval.size()});
         } else {
           if (h->rank != 0) continue;
           lc = A0l + (c - A0g);
@@ -535,13 +535,14 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
         ch_end.push_back(std::min<int64_t>(b + kChunk, (int64_t)cval.size()));
       }
     }
+    if (!by_col.empty()) by_col.resize(((by_col.size() + 4) / 5) * 5);  // whole stars
     cs_ptr.push_back(0);
-    for (auto& v : by_star) {
+    for (auto& v : by_col) {
       for (auto& pr : v) {
-        cs_ak.push_back(pr.first);
+        cs_k.push_back(pr.first);
         cs_e.push_back(pr.second);
       }
-      cs_ptr.push_back((int64_t)cs_ak.size());
+      cs_ptr.push_back((int64_t)cs_k.size());
     }
   }
   h->n_ce = (int64_t)cval.size();
@@ -580,14 +581,14 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   double* d_cval = nullptr;
   int64_t *d_ccol = nullptr, *d_chb = nullptr, *d_che = nullptr, *d_csp = nullptr, *d_cse = nullptr,
           *d_cshi = nullptr, *d_cshe = nullptr;
-  int32_t *d_chr = nullptr, *d_csak = nullptr, *d_cshk = nullptr;
+  int32_t *d_chr = nullptr, *d_csk = nullptr, *d_cshk = nullptr;
   AL(d_cval, h->n_ce);
   AL(d_ccol, h->n_ce);
   AL(d_chr, ch_row.size());
   AL(d_chb, ch_row.size());
   AL(d_che, ch_row.size());
   AL(d_csp, cs_ptr.size());
-  AL(d_csak, cs_ak.size());
+  AL(d_csk, cs_k.size());
   AL(d_cse, cs_e.size());
   AL(d_cshi, csh_idx.size());
   AL(d_cshk, csh_k.size());
@@ -608,7 +609,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
             up(d_chb, ch_beg.data(), sizeof(int64_t) * ch_beg.size()) &&
             up(d_che, ch_end.data(), sizeof(int64_t) * ch_end.size()) &&
             up(d_csp, cs_ptr.data(), sizeof(int64_t) * cs_ptr.size()) &&
-            up(d_csak, cs_ak.data(), sizeof(int32_t) * cs_ak.size()) &&
+            up(d_csk, cs_k.data(), sizeof(int32_t) * cs_k.size()) &&
             up(d_cse, cs_e.data(), sizeof(int64_t) * cs_e.size()) &&
             up(d_cshi, csh_idx.data(), sizeof(int64_t) * csh_idx.size()) &&
             up(d_cshk, csh_k.data(), sizeof(int32_t) * csh_k.size()) &&
@@ -623,7 +624,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   S.G0 = S.I0 + n_instr; S.n_glob = n_glob; S.n_constr = (int32_t)nc;
   S.cval = d_cval; S.ccol = d_ccol; S.n_ce = h->n_ce;
   S.ch_row = d_chr; S.ch_beg = d_chb; S.ch_end = d_che; S.n_chunks = (int64_t)ch_row.size();
-  S.n_cs = cs_ptr.empty() ? 0 : (int64_t)cs_ptr.size() - 1; S.cs_ptr = d_csp; S.cs_ak = d_csak; S.cs_e = d_cse;
+  S.n_cs = cs_ptr.empty() ? 0 : ((int64_t)cs_ptr.size() - 1) / 5; S.cs_ptr = d_csp; S.cs_k = d_csk; S.cs_e = d_cse;
   S.n_csh = (int64_t)csh_idx.size(); S.csh_idx = d_cshi; S.csh_k = d_cshk; S.csh_e = d_cshe;
 
   // zero-initialised state
@@ -687,45 +688,44 @@ int lsqr_set_system(lsqr_t h, const double* vals, const int64_t* mA, const int64
   GUARD(h);
   if (!vals || !mA || !mT || !iC || !b) return LSQR_EINVAL;
   const int64_t n = h->n_loc_rows;
-  std::vector<IdxRec> rec(std::max<int64_t>(n, 1));
-  for (int64_t s = 0; s < h->n_loc_stars; ++s) {
-    for (int64_t i = h->star_ptr_h[s]; i < h->star_ptr_h[s + 1]; ++i) {
-      if (mA[i] != 5 * (h->star_begin + s))
-        return fail(h, LSQR_EUNSORTED, "row %lld: matrixIndexAstro %lld != 5*star %lld", (long long)i,
-                    (long long)mA[i], (long long)(h->star_begin + s));
-      const int64_t k0 = mT[i] - h->A0g;
-      if (k0 < 0 || k0 > h->n_axis - 4) return fail(h, LSQR_EINVAL, "row %lld: matrixIndexAtt out of range", (long long)i);
-      uint32_t ic[6];
-      for (int j = 0; j < 6; ++j) {
-        const int64_t c = iC[i * 6 + j] - h->I0g;
-        if (c < 0 || c >= h->n_instr) return fail(h, LSQR_EINVAL, "row %lld: instrCol out of range", (long long)i);
-        ic[j] = (uint32_t)c;
-      }
-      rec[i].k0 = (int32_t)k0;
-      rec[i].ic01 = ic[0] | (ic[1] << 16);
-      rec[i].ic23 = ic[2] | (ic[3] << 16);
-      rec[i].ic45 = ic[4] | (ic[5] << 16);
-    }
+  // staging for the device-side conversion (paper layout -> lane-major values + 16-B index records), allocated
+  // once: kIngestRows rows of [24 values | mA | mT | 6 instrCol]
+  constexpr int64_t kIngestRows = 1 << 18;
+  if (!h->ingest) {
+    int rc = dalloc(h, &h->ingest, kIngestRows * (kSlots + 8) + 4);
+    if (rc) return rc;
   }
-  // paper slot order -> lane-major device order (position 6j + t holds slot_of(t, j)), in row blocks
+  double* sv = h->ingest;
+  int64_t* smA = reinterpret_cast<int64_t*>(sv + kIngestRows * kSlots);
+  int64_t* smT = smA + kIngestRows;
+  int64_t* siC = smT + kIngestRows;
+  unsigned long long* err = reinterpret_cast<unsigned long long*>(siC + kIngestRows * 6);
   enter(h);
   CKR(reset_precond(h));
-  {
-    const int64_t blk = 1 << 16;
-    std::vector<double> tmp(std::max<int64_t>(std::min(n, blk), 1) * kSlots);
-    for (int64_t r0 = 0; r0 < n; r0 += blk) {
-      const int64_t nb = std::min(blk, n - r0);
-      for (int64_t i = 0; i < nb; ++i)
-        for (int p = 0; p < kSlots; ++p) tmp[i * kSlots + p] = vals[(r0 + i) * kSlots + slot_of(p % 6, p / 6)];
-      CKC(h, cudaMemcpyAsync(h->vals + r0 * kSlots, tmp.data(), sizeof(double) * kSlots * nb,
-                             cudaMemcpyHostToDevice, h->s));
-      CKC(h, cudaStreamSynchronize(h->s));
-    }
+  const unsigned long long err0[2] = {~0ull, 0ull};
+  CKC(h, cudaMemcpyAsync(err, err0, sizeof err0, cudaMemcpyHostToDevice, h->s));
+  for (int64_t r0 = 0; r0 < n; r0 += kIngestRows) {
+    const int64_t nb = std::min(kIngestRows, n - r0);
+    CKC(h, cudaMemcpyAsync(sv, vals + r0 * kSlots, sizeof(double) * kSlots * nb, cudaMemcpyHostToDevice, h->s));
+    CKC(h, cudaMemcpyAsync(smA, mA + r0, sizeof(int64_t) * nb, cudaMemcpyHostToDevice, h->s));
+    CKC(h, cudaMemcpyAsync(smT, mT + r0, sizeof(int64_t) * nb, cudaMemcpyHostToDevice, h->s));
+    CKC(h, cudaMemcpyAsync(siC, iC + r0 * 6, sizeof(int64_t) * 6 * nb, cudaMemcpyHostToDevice, h->s));
+    CKL(h, launch_ingest(sv, smA, smT, siC, r0, nb, h->star_ptr, h->n_loc_stars, h->star_begin, h->A0g, h->I0g,
+                         h->n_axis, h->n_instr, h->vals, h->idx, err, h->s), "ingest");
   }
-  CKC(h, cudaMemcpyAsync(h->idx, rec.data(), sizeof(IdxRec) * n, cudaMemcpyHostToDevice, h->s));
   CKC(h, cudaMemcpyAsync(h->u, b, sizeof(double) * n, cudaMemcpyHostToDevice, h->s));
-  CKC(h, cudaStreamSynchronize(h->s));  // rec is a temporary
+  unsigned long long errh[2];
+  CKC(h, cudaMemcpyAsync(errh, err, sizeof errh, cudaMemcpyDeviceToHost, h->s));
+  CKC(h, cudaStreamSynchronize(h->s));  // host buffers may be reused on return
   leave(h);
+  if (errh[1] != 0) {
+    h->have_system = false;
+    h->b_valid = false;
+    return fail(h, errh[1] == 1 ? LSQR_EUNSORTED : LSQR_EINVAL,
+                errh[1] == 1 ? "row %llu: matrixIndexAstro is not 5*star (rows must be grouped by star in order)"
+                             : "row %llu: attitude or instrumental column out of range",
+                errh[0] - 1);
+  }
   h->have_system = true;
   h->b_valid = true;
   h->initialized = false;

@@ -65,8 +65,8 @@ struct SysView {
   int64_t n_ce;
   // aprod1 constraint dot chunks (each within one row): row, begin, end into cval/ccol
   const int32_t* ch_row; const int64_t* ch_beg; const int64_t* ch_end; int64_t n_chunks;
-  // astro constraint entries grouped by local star (CSC by star): stars [0, n_cs)
-  int64_t n_cs; const int64_t* cs_ptr; const int32_t* cs_ak; const int64_t* cs_e;  // ak = a | (k << 8)
+  // astro constraint entries grouped by local astro column (CSC): columns [0, 5 n_cs) of stars [0, n_cs)
+  int64_t n_cs; const int64_t* cs_ptr; const int32_t* cs_k; const int64_t* cs_e;  // row k, entry index
   // shared-column constraint entries: shared index, constraint row, entry index
   int64_t n_csh; const int64_t* csh_idx; const int32_t* csh_k; const int64_t* csh_e;
 };
@@ -87,6 +87,11 @@ struct GenArgs {
 // All return cudaGetLastError() of the launch.
 cudaError_t launch_generate(const GenArgs& g, double* vals, IdxRec* idx, const int64_t* star_ptr, int64_t n_rows,
                             int64_t n_stars_loc, double* b, cudaStream_t s);
+// lsqr_set_system: host-layout chunk -> device layout with validation (err: [1 + first bad row (min), kind])
+cudaError_t launch_ingest(const double* sv, const int64_t* smA, const int64_t* smT, const int64_t* siC, int64_t row0,
+                          int64_t nrows, const int64_t* star_ptr, int64_t n_stars_loc, int64_t star_begin,
+                          int64_t A0g, int64_t I0g, int64_t n_axis, int64_t n_instr, double* vals, IdxRec* idx,
+                          unsigned long long* err, cudaStream_t s);
 cudaError_t launch_aprod1(int mode, const SysView& S, int grid, const double* x, double* y, double* part,
                           double* cpart, const DevState* st, cudaStream_t s);
 cudaError_t launch_aprod2(int mode, const SysView& S, int grid, const double* y, const double* ucn, double* xv,

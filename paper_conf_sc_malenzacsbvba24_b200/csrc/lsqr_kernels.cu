@@ -466,13 +466,16 @@ __global__ void __launch_bounds__(kThreads, 1)
     z1 += __shfl_xor_sync(0xffffffffu, z1, 16);
     if (lane < 4) {
       if (star < S.n_cs) {  // constraint entries on this star's astro columns (after all rows, as O-AP2)
-        for (int64_t e = S.cs_ptr[star]; e < S.cs_ptr[star + 1]; ++e) {
-          const int ak = S.cs_ak[e], a = ak & 0xff, kk = ak >> 8;
+        const int64_t c0 = 5 * star + j;
+        for (int64_t e = S.cs_ptr[c0]; e < S.cs_ptr[c0 + 1]; ++e) {
           const double cv = S.cval[S.cs_e[e]];
-          const double c = MODE == AP2_COLNORM ? cv * cv : cv * ucn[kk];
-          if (a == j) z0 += c;
-          if (j == 0 && a == 4) z1 += c;
+          z0 += MODE == AP2_COLNORM ? cv * cv : cv * ucn[S.cs_k[e]];
         }
+        if (j == 0)
+          for (int64_t e = S.cs_ptr[5 * star + 4]; e < S.cs_ptr[5 * star + 5]; ++e) {
+            const double cv = S.cval[S.cs_e[e]];
+            z1 += MODE == AP2_COLNORM ? cv * cv : cv * ucn[S.cs_k[e]];
+          }
       }
       double* xc = xv + 5 * star;
       if (MODE == AP2_LSQR) {
@@ -821,14 +824,8 @@ __global__ void __launch_bounds__(kRedThreads)
   double a2 = 0.0;
   for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < na; c += (int64_t)gridDim.x * blockDim.x) {
     double z = zA[c];
-    const int64_t star = c / 5;
-    if (star < S.n_cs) {
-      const int a = (int)(c - 5 * star);
-      for (int64_t e = S.cs_ptr[star]; e < S.cs_ptr[star + 1]; ++e) {
-        const int ak = S.cs_ak[e];
-        if ((ak & 0xff) == a) z += S.cval[S.cs_e[e]] * uc[ak >> 8];
-      }
-    }
+    if (c < 5 * S.n_cs)
+      for (int64_t e = S.cs_ptr[c]; e < S.cs_ptr[c + 1]; ++e) z += S.cval[S.cs_e[e]] * uc[S.cs_k[e]];
     const double vn = z * ib - beta * v[c];
     v[c] = vn;
     a2 = fma(vn, vn, a2);
@@ -1175,6 +1172,62 @@ static int vec_grid(int64_t n, int maxb) {
   int64_t b = (n + kRedThreads - 1) / kRedThreads;
   if (b < 1) b = 1;
   return (int)(b < maxb ? b : maxb);
+}
+
+
+// ------------------------------------------------------------------------------------------------ ingest (set_system)
+// Converts a chunk of host-layout rows (paper slot order, int64 global column indices) into the device
+// layout (lane-major values, 16-B index record), validating the star grouping and index ranges.  err[0] receives
+// (min) 1 + offending row and err[1] the kind (1 unsorted, 2 range) on failure.
+__global__ void k_ingest(const double* __restrict__ sv, const int64_t* __restrict__ smA,
+                         const int64_t* __restrict__ smT, const int64_t* __restrict__ siC, int64_t row0, int64_t nrows,
+                         const int64_t* __restrict__ star_ptr, int64_t n_stars_loc, int64_t star_begin, int64_t A0g,
+                         int64_t I0g, int64_t n_axis, int64_t n_instr, double* __restrict__ vals,
+                         IdxRec* __restrict__ idx, unsigned long long* __restrict__ err) {
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < nrows; q += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t li = row0 + q;
+    int64_t lo = 0, hi = n_stars_loc;  // star_ptr[lo] <= li < star_ptr[hi]
+    while (hi - lo > 1) {
+      const int64_t mid = (lo + hi) >> 1;
+      if (star_ptr[mid] <= li) lo = mid; else hi = mid;
+    }
+    int kind = 0;
+    if (smA[q] != 5 * (star_begin + lo)) kind = 1;
+    const int64_t k0 = smT[q] - A0g;
+    if (k0 < 0 || k0 > n_axis - 4) kind = kind ? kind : 2;
+    uint32_t ic[6];
+#pragma unroll
+    for (int jj = 0; jj < 6; ++jj) {
+      const int64_t c = siC[q * 6 + jj] - I0g;
+      if (c < 0 || c >= n_instr) kind = kind ? kind : 2;
+      ic[jj] = (uint32_t)(c & 0xffff);
+    }
+    if (kind) {
+      atomicMin(err, (unsigned long long)(li + 1));
+      atomicMax(err + 1, (unsigned long long)kind);
+      continue;
+    }
+    IdxRec rec;
+    rec.k0 = (int32_t)k0;
+    rec.ic01 = ic[0] | (ic[1] << 16);
+    rec.ic23 = ic[2] | (ic[3] << 16);
+    rec.ic45 = ic[4] | (ic[5] << 16);
+    idx[li] = rec;
+    const double* src = sv + q * kSlots;
+    double* dst = vals + li * kSlots;
+#pragma unroll
+    for (int pp = 0; pp < kSlots; ++pp) dst[pp] = src[slot_of(pp % 6, pp / 6)];
+  }
+}
+
+cudaError_t launch_ingest(const double* sv, const int64_t* smA, const int64_t* smT, const int64_t* siC, int64_t row0,
+                          int64_t nrows, const int64_t* star_ptr, int64_t n_stars_loc, int64_t star_begin,
+                          int64_t A0g, int64_t I0g, int64_t n_axis, int64_t n_instr, double* vals, IdxRec* idx,
+                          unsigned long long* err, cudaStream_t s) {
+  if (nrows == 0) return cudaSuccess;
+  k_ingest<<<vec_grid(nrows, 148 * 8), kRedThreads, 0, s>>>(sv, smA, smT, siC, row0, nrows, star_ptr, n_stars_loc,
+                                                            star_begin, A0g, I0g, n_axis, n_instr, vals, idx, err);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_generate(const GenArgs& g, double* vals, IdxRec* idx, const int64_t* star_ptr, int64_t n_rows,

@@ -335,3 +335,35 @@ def test_lsqr_C2_full_vs_oracle(avu, fused):
     assert abs(out["r1norm"] - ro["r1norm"]) <= 1e-10 * ro["r1norm"]
     assert rel(out["x"], ro["x"]) <= 1e-9
     s.close()
+
+
+def test_set_system_roundtrip_and_validation(avu):
+    """lsqr_set_system (host paper layout -> device layout, validated on the device) round-trips bit-exactly and
+    rejects rows that are not grouped by star (LSQR_EUNSORTED) or carry out-of-range columns (LSQR_EINVAL)."""
+    w = W.micro(n_stars=60, obs=30, n_ext=5, seed=31)
+    S = oracle.System(w)
+    s = avu.Solver(w.n_stars, w.n_obs, w.n_att, w.n_instr, w.n_glob, obs_per_star=S.counts,
+                   constraints=(S.c_ptr, S.c_col, S.c_val))
+    s.set_system(S.vals, S.mA, S.mT, S.iC, S.b)
+    g = s.get_system()
+    for k in ("vals", "mA", "mT", "iC", "b"):
+        assert np.array_equal(g[k], getattr(S, k)), k
+    # products on the uploaded system equal the oracle's
+    import torch
+    x = np.random.default_rng(0).standard_normal(S.n_cols)
+    y = torch.zeros(S.m_local, dtype=torch.float64, device="cuda")
+    s.aprod1(torch.tensor(x, device="cuda"), y)
+    yr = np.zeros(S.m_local); S.aprod1(x, yr)
+    assert np.allclose(y.cpu().numpy(), yr, rtol=1e-13, atol=1e-13)
+    bad = S.mA.copy(); bad[[10, 40]] = bad[[40, 10]]
+    with pytest.raises(avu.LsqrError) as ei:
+        s.set_system(S.vals, bad, S.mT, S.iC, S.b)
+    assert ei.value.status == -6
+    bad_t = S.mT.copy(); bad_t[5] = S.A0 + w.n_att
+    with pytest.raises(avu.LsqrError) as ei:
+        s.set_system(S.vals, S.mA, bad_t, S.iC, S.b)
+    assert ei.value.status == -1
+    s.set_system(S.vals, S.mA, S.mT, S.iC, S.b)  # a valid upload re-arms the handle
+    out = s.solve(itn_limit=50, atol=0, btol=0, conlim=0, fixed_count=True)
+    assert out["itn"] == 50
+    s.close()
