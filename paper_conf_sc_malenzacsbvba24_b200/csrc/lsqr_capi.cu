@@ -626,6 +626,11 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   S.ch_row = d_chr; S.ch_beg = d_chb; S.ch_end = d_che; S.n_chunks = (int64_t)ch_row.size();
   S.n_cs = cs_ptr.empty() ? 0 : ((int64_t)cs_ptr.size() - 1) / 5; S.cs_ptr = d_csp; S.cs_k = d_csk; S.cs_e = d_cse;
   S.n_csh = (int64_t)csh_idx.size(); S.csh_idx = d_cshi; S.csh_k = d_cshk; S.csh_e = d_cshe;
+  {  // bank-grouped instrumental slots only when every row kernel keeps the instrumental slice in shared memory
+    InstrPerm probe;
+    probe.init(n_instr, true);
+    S.ip.init(n_instr, probe.slots() <= kInstrSmemMax);
+  }
 
   // zero-initialised state
   if (launch_fill(h->zsh, h->n_sh + 8, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
@@ -672,6 +677,7 @@ int lsqr_generate(lsqr_t h, const lsqr_gen_params* p) {
   enter(h);
   CKR(reset_precond(h));
   GenArgs g;
+  g.ip = h->S.ip;
   g.seed = p->seed; g.b_mode = p->b_mode; g.noise = p->noise;
   g.row_begin_global = h->row_begin; g.star_begin_global = h->star_begin;
   g.n_stars_global = h->n_stars; g.n_att = h->n_att; g.n_instr = h->n_instr; g.n_glob = h->n_glob;
@@ -711,7 +717,7 @@ int lsqr_set_system(lsqr_t h, const double* vals, const int64_t* mA, const int64
     CKC(h, cudaMemcpyAsync(smT, mT + r0, sizeof(int64_t) * nb, cudaMemcpyHostToDevice, h->s));
     CKC(h, cudaMemcpyAsync(siC, iC + r0 * 6, sizeof(int64_t) * 6 * nb, cudaMemcpyHostToDevice, h->s));
     CKL(h, launch_ingest(sv, smA, smT, siC, r0, nb, h->star_ptr, h->n_loc_stars, h->star_begin, h->A0g, h->I0g,
-                         h->n_axis, h->n_instr, h->vals, h->idx, err, h->s), "ingest");
+                         h->n_axis, h->n_instr, h->S.ip, h->vals, h->idx, err, h->s), "ingest");
   }
   CKC(h, cudaMemcpyAsync(h->u, b, sizeof(double) * n, cudaMemcpyHostToDevice, h->s));
   unsigned long long errh[2];
@@ -749,6 +755,8 @@ int lsqr_get_system(lsqr_t h, double* vals, int64_t* mA, int64_t* mT, int64_t* i
   }
   if (b) CKC(h, cudaMemcpy(b, h->u, sizeof(double) * n, cudaMemcpyDeviceToHost));
   if (mA || mT || iC) {
+    std::vector<int64_t> inv(std::max<int64_t>(h->S.ip.slots(), 1), 0);  // shared-memory slot -> column
+    for (int64_t c = 0; c < h->n_instr; ++c) inv[h->S.ip.fwd(c)] = c;
     std::vector<IdxRec> rec(std::max<int64_t>(n, 1));
     CKC(h, cudaMemcpy(rec.data(), h->idx, sizeof(IdxRec) * n, cudaMemcpyDeviceToHost));
     for (int64_t s = 0; s < h->n_loc_stars; ++s)
@@ -757,7 +765,7 @@ int lsqr_get_system(lsqr_t h, double* vals, int64_t* mA, int64_t* mT, int64_t* i
         if (mT) mT[i] = h->A0g + rec[i].k0;
         if (iC) {
           const uint32_t w3[3] = {rec[i].ic01, rec[i].ic23, rec[i].ic45};
-          for (int j = 0; j < 6; ++j) iC[i * 6 + j] = h->I0g + ((w3[j / 2] >> ((j & 1) * 16)) & 0xffff);
+          for (int j = 0; j < 6; ++j) iC[i * 6 + j] = h->I0g + inv[(w3[j / 2] >> ((j & 1) * 16)) & 0xffff];
         }
       }
   }

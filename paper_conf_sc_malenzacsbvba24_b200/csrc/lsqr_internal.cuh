@@ -17,7 +17,7 @@ constexpr int kStageBytes = kRows * (kSlots * 8 + 16);                  // 3328 
 constexpr int kRingBytes = kWarpsPerCta * kStages * kStageBytes;        // 159,744 B per CTA
 constexpr int kBarBytes = kWarpsPerCta * kStages * 8;                   // mbarriers
 constexpr int kRedThreads = 256;     // small reduction / vector kernels
-constexpr int kInstrSmemMax = 8192;  // n_instr above this -> instrumental scatter goes to L2 REDs (no smem)
+constexpr int kInstrSmemMax = 7680;  // n_instr above this -> instrumental gathers/scatter use global memory (L2)
 constexpr int kMaxConstr = 64;       // constraint rows handled by the one-block beta kernel
 constexpr int kMaxChunksSmem = 1024; // constraint chunk partials staged in shared memory by k_beta
 
@@ -36,6 +36,38 @@ struct __align__(16) IdxRec {
   uint32_t ic01, ic23, ic45;  // instrCol[j] in 16-bit halves (j even: low half)
 };
 static_assert(sizeof(IdxRec) == 16, "IdxRec must be 16 bytes");
+
+// Shared-memory slot of instrumental column c (device-internal; stored in IdxRec).  With the generator's structure
+// (row j-th instrumental column in group j of g = n_instr/6 columns), the 8 lanes that touch group j (< 4) in one
+// warp instruction get their own 4 of the 16 bank pairs, and groups 4 / 5 (touched together) get 8 each, which cuts
+// bank conflicts of the instrumental gathers and CAS updates.  Identity when disabled (n_instr % 6 != 0 or the
+// instrumental slice is not kept in shared memory).
+struct InstrPerm {
+  int64_t n = 0, g = 0, oa = 0;
+  bool on = false;
+  __host__ __device__ void init(int64_t n_instr, bool enable) {
+    n = n_instr;
+    on = enable && n_instr % 6 == 0 && n_instr >= 6;
+    g = on ? n_instr / 6 : 0;
+    oa = on ? 16 * ((g + 3) / 4) : 0;
+  }
+  __host__ __device__ int64_t slots() const { return on ? oa + 16 * ((g + 7) / 8) : n; }
+  __host__ __device__ int64_t fwd(int64_t c) const {
+    if (!on) return c;
+    const int64_t grp = c / g, t = c - grp * g;
+    if (grp < 4) return 16 * (t >> 2) + 4 * grp + (t & 3);
+    return oa + 16 * (t >> 3) + 8 * (grp - 4) + (t & 7);
+  }
+  __host__ __device__ int64_t inv(int64_t p) const {  // slot -> column
+    if (!on) return p;
+    if (p < oa) {
+      const int64_t b = p >> 4, w = p & 15;
+      return (w >> 2) * g + 4 * b + (w & 3);
+    }
+    const int64_t q = p - oa, b = q >> 4, w = q & 15;
+    return (4 + (w >> 3)) * g + 8 * b + (w & 7);
+  }
+};
 
 // LSQR scalar state kept on the device (Paige-Saunders scalars) + control flags.
 struct DevState {
@@ -69,12 +101,14 @@ struct SysView {
   int64_t n_cs; const int64_t* cs_ptr; const int32_t* cs_k; const int64_t* cs_e;  // row k, entry index
   // shared-column constraint entries: shared index, constraint row, entry index
   int64_t n_csh; const int64_t* csh_idx; const int32_t* csh_k; const int64_t* csh_e;
+  InstrPerm ip;  // IdxRec instrumental fields hold ip.fwd(column); shared-memory arrays have ip.slots() entries
 };
 
 enum { AP1_LSQR = 0, AP1_PLAIN = 1 };
 enum { AP2_LSQR = 0, AP2_PLAIN = 1, AP2_COLNORM = 2 };
 
 struct GenArgs {
+  InstrPerm ip;
   uint64_t seed;
   int32_t b_mode;
   double noise;
@@ -90,8 +124,8 @@ cudaError_t launch_generate(const GenArgs& g, double* vals, IdxRec* idx, const i
 // lsqr_set_system: host-layout chunk -> device layout with validation (err: [1 + first bad row (min), kind])
 cudaError_t launch_ingest(const double* sv, const int64_t* smA, const int64_t* smT, const int64_t* siC, int64_t row0,
                           int64_t nrows, const int64_t* star_ptr, int64_t n_stars_loc, int64_t star_begin,
-                          int64_t A0g, int64_t I0g, int64_t n_axis, int64_t n_instr, double* vals, IdxRec* idx,
-                          unsigned long long* err, cudaStream_t s);
+                          int64_t A0g, int64_t I0g, int64_t n_axis, int64_t n_instr, InstrPerm ip, double* vals,
+                          IdxRec* idx, unsigned long long* err, cudaStream_t s);
 cudaError_t launch_aprod1(int mode, const SysView& S, int grid, const double* x, double* y, double* part,
                           double* cpart, const DevState* st, cudaStream_t s);
 cudaError_t launch_aprod2(int mode, const SysView& S, int grid, const double* y, const double* ucn, double* xv,

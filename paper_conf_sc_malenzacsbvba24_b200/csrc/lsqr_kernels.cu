@@ -85,9 +85,9 @@ __global__ void k_generate(GenArgs g, double* __restrict__ vals, IdxRec* __restr
     for (int j = 0; j < 6; ++j) ic[j] = (uint32_t)(j * grp + (int64_t)(g_hash(g.seed, 3, i, j) % (uint64_t)grp));
     IdxRec rec;
     rec.k0 = (int32_t)k0;
-    rec.ic01 = ic[0] | (ic[1] << 16);
-    rec.ic23 = ic[2] | (ic[3] << 16);
-    rec.ic45 = ic[4] | (ic[5] << 16);
+    rec.ic01 = (uint32_t)g.ip.fwd(ic[0]) | ((uint32_t)g.ip.fwd(ic[1]) << 16);
+    rec.ic23 = (uint32_t)g.ip.fwd(ic[2]) | ((uint32_t)g.ip.fwd(ic[3]) << 16);
+    rec.ic45 = (uint32_t)g.ip.fwd(ic[4]) | ((uint32_t)g.ip.fwd(ic[5]) << 16);
     idx[li] = rec;
     double v[kSlots];
 #pragma unroll
@@ -240,8 +240,8 @@ __device__ __forceinline__ void stage_row(const unsigned char* stg, int lr, int 
 __device__ __forceinline__ int64_t col_of(const SysView& S, int t, int j, int64_t star, const IdxRec& r) {
   if (t == 0) return 5 * star + j;
   if (t <= 3) return S.A0 + (int64_t)(t - 1) * S.n_axis + r.k0 + j;
-  if (t == 4) return S.I0 + ic_of(r, j);
-  return j == 0 ? 5 * star + 4 : (j == 3 ? S.G0 : S.I0 + ic_of(r, 3 + j));
+  if (t == 4) return S.I0 + S.ip.inv(ic_of(r, j));
+  return j == 0 ? 5 * star + 4 : (j == 3 ? S.G0 : S.I0 + S.ip.inv(ic_of(r, 3 + j)));
 }
 
 // lane-local star of a row (rows are grouped by star, visited in increasing order): s / bound cached in registers
@@ -321,7 +321,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   // the instrumental slice of x (<= 64 KB) is staged in shared memory: its gathers are random and L1-hostile
   double* sh_x = reinterpret_cast<double*>(dsm + kRingBytes + kBarBytes);
   if (SMEM_INSTR) {
-    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_x[i] = x[S.I0 + i];
+    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_x[S.ip.fwd(i)] = x[S.I0 + i];
     __syncthreads();
   }
   const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2, wid = threadIdx.x >> 5;
@@ -425,7 +425,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   if (MODE == AP2_LSQR && (st->halted || !st->beta_pos)) return;
   double* sh_instr = reinterpret_cast<double*>(dsm + kRingBytes + kBarBytes);
   if (SMEM_INSTR) {
-    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_instr[i] = 0.0;
+    for (int64_t i = threadIdx.x; i < S.ip.slots(); i += blockDim.x) sh_instr[i] = 0.0;
     __syncthreads();
   }
   const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2, wid = threadIdx.x >> 5;
@@ -598,7 +598,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   if (SMEM_INSTR) {
     __syncthreads();
     for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
-      const double v = sh_instr[i];
+      const double v = sh_instr[S.ip.fwd(i)];
       if (v != 0.0) atomicAdd(zsh + S.n_att + i, v);
     }
   }
@@ -626,14 +626,17 @@ __global__ void __launch_bounds__(kThreads, 1)
   extern __shared__ __align__(128) unsigned char dsm[];
   if (st->halted) return;
   // shared memory: [ring | mbarriers | v_instr (n_instr) + v_glob | z_instr accumulator (n_instr)]
+  const int64_t nsl = S.ip.slots();
   double* sh_x = reinterpret_cast<double*>(dsm + FRing::kBytes + FRing::kBars);
-  double* sh_z = sh_x + S.n_instr + 2;
+  double* sh_z = sh_x + nsl + 2;
   if (SMEM_INSTR) {
-    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
-      sh_x[i] = x[S.I0 + i];
+    for (int64_t i = threadIdx.x; i < nsl; i += blockDim.x) {
+      sh_x[i] = 0.0;
       sh_z[i] = 0.0;
     }
-    if (threadIdx.x == 0) sh_x[S.n_instr] = S.n_glob ? x[S.G0] : 0.0;
+    __syncthreads();
+    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_x[S.ip.fwd(i)] = x[S.I0 + i];
+    if (threadIdx.x == 0) sh_x[nsl] = S.n_glob ? x[S.G0] : 0.0;
     __syncthreads();
   }
   const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2, wid = threadIdx.x >> 5;
@@ -719,7 +722,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     const int k0 = rec.k0;
     const uint32_t i4 = ic4_of(rec, j);
-    const uint32_t i5 = (j == 3) ? (uint32_t)S.n_instr : ic5_of(rec, j);
+    const uint32_t i5 = (j == 3) ? (uint32_t)nsl : ic5_of(rec, j);
     const double g1 = __ldg(xatt0 + k0), g2 = __ldg(xatt1 + k0), g3 = __ldg(xatt2 + k0);
     double g4, g5;
     if (SMEM_INSTR) {
@@ -806,7 +809,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   if (SMEM_INSTR) {
     __syncthreads();
     for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
-      const double vv = sh_z[i];
+      const double vv = sh_z[S.ip.fwd(i)];
       if (vv != 0.0) atomicAdd(zsh + S.n_att + i, vv);
     }
   }
@@ -1182,7 +1185,7 @@ static int vec_grid(int64_t n, int maxb) {
 __global__ void k_ingest(const double* __restrict__ sv, const int64_t* __restrict__ smA,
                          const int64_t* __restrict__ smT, const int64_t* __restrict__ siC, int64_t row0, int64_t nrows,
                          const int64_t* __restrict__ star_ptr, int64_t n_stars_loc, int64_t star_begin, int64_t A0g,
-                         int64_t I0g, int64_t n_axis, int64_t n_instr, double* __restrict__ vals,
+                         int64_t I0g, int64_t n_axis, int64_t n_instr, InstrPerm ip, double* __restrict__ vals,
                          IdxRec* __restrict__ idx, unsigned long long* __restrict__ err) {
   for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < nrows; q += (int64_t)gridDim.x * blockDim.x) {
     const int64_t li = row0 + q;
@@ -1200,7 +1203,7 @@ __global__ void k_ingest(const double* __restrict__ sv, const int64_t* __restric
     for (int jj = 0; jj < 6; ++jj) {
       const int64_t c = siC[q * 6 + jj] - I0g;
       if (c < 0 || c >= n_instr) kind = kind ? kind : 2;
-      ic[jj] = (uint32_t)(c & 0xffff);
+      ic[jj] = (uint32_t)(ip.fwd(c < 0 || c >= n_instr ? 0 : c) & 0xffff);
     }
     if (kind) {
       atomicMin(err, (unsigned long long)(li + 1));
@@ -1222,11 +1225,12 @@ __global__ void k_ingest(const double* __restrict__ sv, const int64_t* __restric
 
 cudaError_t launch_ingest(const double* sv, const int64_t* smA, const int64_t* smT, const int64_t* siC, int64_t row0,
                           int64_t nrows, const int64_t* star_ptr, int64_t n_stars_loc, int64_t star_begin,
-                          int64_t A0g, int64_t I0g, int64_t n_axis, int64_t n_instr, double* vals, IdxRec* idx,
-                          unsigned long long* err, cudaStream_t s) {
+                          int64_t A0g, int64_t I0g, int64_t n_axis, int64_t n_instr, InstrPerm ip, double* vals,
+                          IdxRec* idx, unsigned long long* err, cudaStream_t s) {
   if (nrows == 0) return cudaSuccess;
   k_ingest<<<vec_grid(nrows, 148 * 8), kRedThreads, 0, s>>>(sv, smA, smT, siC, row0, nrows, star_ptr, n_stars_loc,
-                                                            star_begin, A0g, I0g, n_axis, n_instr, vals, idx, err);
+                                                            star_begin, A0g, I0g, n_axis, n_instr, ip, vals, idx,
+                                                            err);
   return cudaGetLastError();
 }
 
@@ -1240,11 +1244,11 @@ cudaError_t launch_generate(const GenArgs& g, double* vals, IdxRec* idx, const i
 template <int MODE, bool SM>
 static cudaError_t ap1(const SysView& S, int grid, const double* x, double* y, double* part, double* cpart,
                        const DevState* st, cudaStream_t s) {
-  const size_t smem = kRingBytes + kBarBytes + (SM ? (size_t)S.n_instr * sizeof(double) : 0);
+  const size_t smem = kRingBytes + kBarBytes + (SM ? (size_t)S.ip.slots() * sizeof(double) : 0);
   static bool attr_set = false;
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(k_aprod1<MODE, SM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)(kRingBytes + kBarBytes + (SM ? kInstrSmemMax * sizeof(double) : 0)));
+                                         (int)(kRingBytes + kBarBytes + (SM ? (kInstrSmemMax + 64) * sizeof(double) : 0)));
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
@@ -1254,7 +1258,7 @@ static cudaError_t ap1(const SysView& S, int grid, const double* x, double* y, d
 
 cudaError_t launch_aprod1(int mode, const SysView& S, int grid, const double* x, double* y, double* part,
                           double* cpart, const DevState* st, cudaStream_t s) {
-  const bool sm = S.n_instr <= kInstrSmemMax;
+  const bool sm = S.ip.slots() <= kInstrSmemMax;
   if (mode == AP1_LSQR) return sm ? ap1<AP1_LSQR, true>(S, grid, x, y, part, cpart, st, s)
                                   : ap1<AP1_LSQR, false>(S, grid, x, y, part, cpart, st, s);
   return sm ? ap1<AP1_PLAIN, true>(S, grid, x, y, part, cpart, st, s)
@@ -1264,11 +1268,11 @@ cudaError_t launch_aprod1(int mode, const SysView& S, int grid, const double* x,
 template <int MODE, bool SM>
 static cudaError_t ap2(const SysView& S, int grid, const double* y, const double* ucn, double* xv, double* zsh,
                        double* part, const DevState* st, int dsc, cudaStream_t s) {
-  size_t smem = kRingBytes + kBarBytes + (SM ? (size_t)S.n_instr * sizeof(double) : 0);
+  size_t smem = kRingBytes + kBarBytes + (SM ? (size_t)S.ip.slots() * sizeof(double) : 0);
   static bool attr_set = false;
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(k_aprod2<MODE, SM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)(kRingBytes + kBarBytes + (SM ? kInstrSmemMax * sizeof(double) : 0)));
+                                         (int)(kRingBytes + kBarBytes + (SM ? (kInstrSmemMax + 64) * sizeof(double) : 0)));
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
@@ -1278,7 +1282,7 @@ static cudaError_t ap2(const SysView& S, int grid, const double* y, const double
 
 cudaError_t launch_aprod2(int mode, const SysView& S, int grid, const double* y, const double* ucn, double* xv,
                           double* zsh, double* part, const DevState* st, int dsc, cudaStream_t s) {
-  const bool sm = S.n_instr <= kInstrSmemMax;
+  const bool sm = S.ip.slots() <= kInstrSmemMax;
   switch (mode) {
     case AP2_LSQR: return sm ? ap2<AP2_LSQR, true>(S, grid, y, ucn, xv, zsh, part, st, dsc, s)
                              : ap2<AP2_LSQR, false>(S, grid, y, ucn, xv, zsh, part, st, dsc, s);
@@ -1321,7 +1325,7 @@ cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* p
 template <bool SM>
 static cudaError_t fz(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh, double* part,
                       double* cpart, const DevState* st, cudaStream_t s) {
-  const size_t smem = FRing::kBytes + FRing::kBars + (SM ? (2 * (size_t)S.n_instr + 2) * sizeof(double) : 0);
+  const size_t smem = FRing::kBytes + FRing::kBars + (SM ? (2 * (size_t)S.ip.slots() + 4) * sizeof(double) : 0);
   static bool attr_set = false;
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(k_fused<SM>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemMaxBytes);
@@ -1334,7 +1338,7 @@ static cudaError_t fz(const SysView& S, int grid, const double* x, double* u, do
 
 cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh,
                          double* part, double* cpart, const DevState* st, cudaStream_t s) {
-  return S.n_instr <= kFusedInstrMax ? fz<true>(S, grid, x, u, zA, zsh, part, cpart, st, s)
+  return S.ip.slots() <= kFusedInstrMax ? fz<true>(S, grid, x, u, zA, zsh, part, cpart, st, s)
                                      : fz<false>(S, grid, x, u, zA, zsh, part, cpart, st, s);
 }
 
