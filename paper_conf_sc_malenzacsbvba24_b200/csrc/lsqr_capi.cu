@@ -94,7 +94,8 @@ struct lsqr_ctx {
   double *vals = nullptr, *u = nullptr, *v = nullptr, *w = nullptr, *x = nullptr, *var = nullptr, *D = nullptr;
   double *zsh = nullptr, *part_rows = nullptr, *part_a2 = nullptr, *cpart = nullptr, *part_sh = nullptr;
   double *zA = nullptr, *part_va = nullptr;
-  double* ingest = nullptr;  // lsqr_set_system staging (lazily allocated)  // fused mode: astro z (A^T u_hat) and alpha^2 partials of k_vastro
+  double* ingest = nullptr;  // lsqr_set_system staging (lazily allocated)
+  double* uc_tmp = nullptr;  // k_post -> k_scalar constraint u_hat hand-over  // fused mode: astro z (A^T u_hat) and alpha^2 partials of k_vastro
   double *part_wa = nullptr, *part_ws = nullptr, *part_g1 = nullptr, *ar1 = nullptr, *uc = nullptr,
          *ucn = nullptr, *crhs = nullptr, *tmp = nullptr, *tmax = nullptr;
   IdxRec* idx = nullptr;
@@ -250,6 +251,17 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
     CKL(h, launch_aprod1(AP1_LSQR, S, h->grid, h->v, h->u, h->part_rows, h->cpart, h->st, s), "aprod1");
   }
   if (ev) cudaEventRecord(ev[1], s);
+  if (fused && !multi) {  // 4 launches: fused rows, post (beta + v' everywhere), scalar, column update
+    if (ev) cudaEventRecord(ev[2], s);
+    CKL(h, launch_post(S, h->v, h->zA, h->zsh, h->part_rows, h->W, h->cpart, h->uc, h->uc_tmp, h->part_va, kG3,
+                       h->st, s), "post");
+    if (ev) cudaEventRecord(ev[3], s);
+    CKL(h, launch_scalar(h->st, h->part_va, kG3, nullptr, 0, h->part_wa, kG3, h->part_ws, kG3, nullptr, nullptr, 0,
+                         h->hflag_dev, s, h->uc_tmp, h->uc, h->ucn, (int)h->n_constr), "scalar");
+    CKL(h, launch_colupdate(h->v, h->w, h->x, h->var, h->n_loc_cols, S.A0, h->part_wa, h->part_ws, kG3, h->st, s),
+        "colupdate");
+    return LSQR_OK;
+  }
   if (!multi) {
     CKL(h, launch_beta(0, S, h->part_rows, h->W, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta");
   } else {
@@ -288,7 +300,7 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   return LSQR_OK;
 }
 
-int kernels_per_iteration(lsqr_t h) { return h->nranks > 1 ? 9 : 6; }  // same count in both modes
+int kernels_per_iteration(lsqr_t h) { return h->nranks > 1 ? 9 : (h->params.fused ? 4 : 6); }
 
 int build_graph(lsqr_t h) {
   if (h->gexec) {
@@ -547,6 +559,23 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   }
   h->n_ce = (int64_t)cval.size();
   h->cval_raw = cval;
+  // shared-column constraint entries as a CSC over [scs_lo, scs_hi) of the shared slice (entry order kept)
+  int64_t scs_lo = 0, scs_hi = 0;
+  std::vector<int64_t> scs_ptr(1, 0), scs_e;
+  std::vector<int32_t> scs_k;
+  if (!csh_idx.empty()) {
+    scs_lo = *std::min_element(csh_idx.begin(), csh_idx.end());
+    scs_hi = *std::max_element(csh_idx.begin(), csh_idx.end()) + 1;
+    std::vector<std::vector<std::pair<int32_t, int64_t>>> by(scs_hi - scs_lo);
+    for (size_t q = 0; q < csh_idx.size(); ++q) by[csh_idx[q] - scs_lo].push_back({csh_k[q], csh_e[q]});
+    for (auto& v : by) {
+      for (auto& pr : v) {
+        scs_k.push_back(pr.first);
+        scs_e.push_back(pr.second);
+      }
+      scs_ptr.push_back((int64_t)scs_k.size());
+    }
+  }
 
   // ---- allocations
   int rc = LSQR_OK;
@@ -567,6 +596,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   AL(h->cpart, std::max<int64_t>((int64_t)ch_row.size(), 1));
   AL(h->part_sh, kG2);
   AL(h->zA, 5 * h->n_loc_stars);
+  AL(h->uc_tmp, kMaxConstr);
   AL(h->part_va, kG3);
   AL(h->part_wa, kG3);
   AL(h->part_ws, kG3);
@@ -593,6 +623,11 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   AL(d_cshi, csh_idx.size());
   AL(d_cshk, csh_k.size());
   AL(d_cshe, csh_e.size());
+  int64_t *d_scsp = nullptr, *d_scse = nullptr;
+  int32_t* d_scsk = nullptr;
+  AL(d_scsp, scs_ptr.size());
+  AL(d_scsk, scs_k.size());
+  AL(d_scse, scs_e.size());
 #undef AL
   if (cudaHostAlloc(&h->hflag, sizeof(int32_t) * 4, cudaHostAllocMapped) != cudaSuccess) return bail(LSQR_ENOMEM);
   h->hflag[0] = 0;
@@ -614,6 +649,9 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
             up(d_cshi, csh_idx.data(), sizeof(int64_t) * csh_idx.size()) &&
             up(d_cshk, csh_k.data(), sizeof(int32_t) * csh_k.size()) &&
             up(d_cshe, csh_e.data(), sizeof(int64_t) * csh_e.size()) &&
+            up(d_scsp, scs_ptr.data(), sizeof(int64_t) * scs_ptr.size()) &&
+            up(d_scsk, scs_k.data(), sizeof(int32_t) * scs_k.size()) &&
+            up(d_scse, scs_e.data(), sizeof(int64_t) * scs_e.size()) &&
             up(h->crhs, crhs.data(), sizeof(double) * nc);
   if (!ok) return bail(LSQR_ECUDA);
 
@@ -626,6 +664,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   S.ch_row = d_chr; S.ch_beg = d_chb; S.ch_end = d_che; S.n_chunks = (int64_t)ch_row.size();
   S.n_cs = cs_ptr.empty() ? 0 : ((int64_t)cs_ptr.size() - 1) / 5; S.cs_ptr = d_csp; S.cs_k = d_csk; S.cs_e = d_cse;
   S.n_csh = (int64_t)csh_idx.size(); S.csh_idx = d_cshi; S.csh_k = d_cshk; S.csh_e = d_cshe;
+  S.scs_lo = scs_lo; S.scs_hi = scs_hi; S.scs_ptr = d_scsp; S.scs_k = d_scsk; S.scs_e = d_scse;
   {  // bank-grouped instrumental slots only when every row kernel keeps the instrumental slice in shared memory
     InstrPerm probe;
     probe.init(n_instr, true);

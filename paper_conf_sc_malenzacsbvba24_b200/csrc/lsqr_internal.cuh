@@ -79,8 +79,9 @@ struct DevState {
   double inv_alpha;  // colupdate: v <- v * inv_alpha when v_pending
   double t1, t2, t3; // x += t1 w ; w = v + t2 w ; d = t3 w
   double rn_tmp;
+  double pb_beta, pb_ib;  // k_post -> k_scalar hand-over (written by k_post block 0, read by k_scalar only)
   int32_t itn, istop, istop_first, itn_limit;
-  int32_t fixed_count, halted, col_enable, v_pending, beta_pos, pad_[3];
+  int32_t fixed_count, halted, col_enable, v_pending, beta_pos, pb_pos, pad_[2];
 };
 
 // Everything a row kernel needs, passed by value.
@@ -102,6 +103,8 @@ struct SysView {
   // shared-column constraint entries: shared index, constraint row, entry index
   int64_t n_csh; const int64_t* csh_idx; const int32_t* csh_k; const int64_t* csh_e;
   InstrPerm ip;  // IdxRec instrumental fields hold ip.fwd(column); shared-memory arrays have ip.slots() entries
+  // shared-column constraint entries grouped by shared column (CSC) over [scs_lo, scs_hi) (rank 0 only)
+  int64_t scs_lo, scs_hi; const int64_t* scs_ptr; const int32_t* scs_k; const int64_t* scs_e;
 };
 
 enum { AP1_LSQR = 0, AP1_PLAIN = 1 };
@@ -150,7 +153,12 @@ cudaError_t launch_add_shared(double* xsh, double* zsh, int64_t n, int mode, cud
 cudaError_t launch_scalar(DevState* st, const double* part_astro, int64_t n_pa, const double* part_sh,
                           int64_t n_ps, const double* part_wa, int64_t n_pwa, const double* part_ws, int64_t n_pws,
                           const double* ar2_alpha2, const double* ar1_wa, int init, int32_t* host_flag,
-                          cudaStream_t s);
+                          cudaStream_t s, const double* post_uc = nullptr, double* uc = nullptr,
+                          double* ucn = nullptr, int nc = 0);
+// single-rank fused mode: beta (recomputed per block) + astro/shared v' + constraint terms in one kernel
+cudaError_t launch_post(const SysView& S, double* v, const double* zA, double* zsh, const double* part_rows,
+                        int64_t n_part, const double* cpart, const double* uc, double* uc_tmp, double* part_a2,
+                        int nblk, DevState* st, cudaStream_t s);
 cudaError_t launch_colupdate(double* v, double* w, double* x, double* var, int64_t n, int64_t A0, double* part_wa,
                              double* part_ws, int nblk, const DevState* st, cudaStream_t s);
 cudaError_t launch_sum_to(const double* part, int64_t n, double* dst, cudaStream_t s);

@@ -43,6 +43,30 @@ __device__ __forceinline__ double ordered_sum(const double* __restrict__ part, i
   return block_sum<NT>(s);
 }
 
+// up to 4 ordered sums at once (one load phase, one reduction phase); results valid in thread 0
+template <int NT>
+__device__ __forceinline__ void ordered_sum4(const double* p0, int64_t n0, const double* p1, int64_t n1,
+                                             const double* p2, int64_t n2, const double* p3, int64_t n3,
+                                             double (&out)[4]) {
+  double a[4] = {0.0, 0.0, 0.0, 0.0};
+  for (int64_t i = threadIdx.x; i < n0; i += NT) a[0] += p0[i];
+  for (int64_t i = threadIdx.x; i < n1; i += NT) a[1] += p1[i];
+  for (int64_t i = threadIdx.x; i < n2; i += NT) a[2] += p2[i];
+  for (int64_t i = threadIdx.x; i < n3; i += NT) a[3] += p3[i];
+  __shared__ double red4[4][NT / 32];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const double v = warp_sum(a[q]);
+    if ((threadIdx.x & 31) == 0) red4[q][threadIdx.x >> 5] = v;
+  }
+  __syncthreads();
+  if (threadIdx.x < 32) {
+#pragma unroll
+    for (int q = 0; q < 4; ++q) out[q] = warp_sum(threadIdx.x < NT / 32 ? red4[q][threadIdx.x] : 0.0);
+  }
+  __syncthreads();
+}
+
 __device__ __forceinline__ uint32_t ic_of(const IdxRec& r, int q) {  // instrCol q (0..5), relative to I0
   uint32_t w = q < 2 ? r.ic01 : (q < 4 ? r.ic23 : r.ic45);
   return (w >> ((q & 1) * 16)) & 0xffffu;
@@ -841,6 +865,97 @@ __global__ void __launch_bounds__(kRedThreads)
       atomicAdd(zsh + S.csh_idx[e], S.cval[S.csh_e[e]] * uc[S.csh_k[e]]);
 }
 
+
+// Single-rank fused mode, after k_fused: beta (every block recomputes it from the deterministic partials; block 0
+// hands it to k_scalar through st->pb_*), then v' = z/beta - beta v on all local columns (astro from zA, shared
+// from z_sh, which is zeroed for the next iteration), constraint terms added per column, alpha^2 partials.
+__global__ void __launch_bounds__(kRedThreads)
+    k_post(SysView S, double* __restrict__ v, const double* __restrict__ zA, double* __restrict__ zsh,
+           const double* __restrict__ part_rows, int64_t n_part, const double* __restrict__ cpart,
+           const double* __restrict__ uc, double* __restrict__ uc_tmp, double* __restrict__ part_a2,
+           DevState* __restrict__ st) {
+  __shared__ double un_sh[kMaxConstr];
+  __shared__ double cd_sh[kMaxConstr];
+  __shared__ double bsh[3];
+  if (st->halted) return;
+  const int nc = S.n_constr;
+  const double b2r = ordered_sum<kRedThreads>(part_rows, n_part);
+  __shared__ double cp_sh[kMaxChunksSmem];
+  __shared__ int32_t cr_sh[kMaxChunksSmem];
+  const int64_t nch = S.n_chunks;
+  const bool in_smem = nch <= kMaxChunksSmem;
+  if (in_smem)
+    for (int64_t c = threadIdx.x; c < nch; c += blockDim.x) {
+      cp_sh[c] = cpart[c];
+      cr_sh[c] = S.ch_row[c];
+    }
+  __syncthreads();
+  if (threadIdx.x < nc) {  // constraint row dots from the chunk partials (chunks are in row order)
+    double d = 0.0;
+    for (int64_t c = 0; c < nch; ++c) {
+      const int rw = in_smem ? cr_sh[c] : S.ch_row[c];
+      if (rw == (int)threadIdx.x) d += in_smem ? cp_sh[c] : cpart[c];
+    }
+    cd_sh[threadIdx.x] = d;
+    un_sh[threadIdx.x] = uc[threadIdx.x];
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const double us = st->u_scale;
+    double b2 = b2r;
+    for (int k = 0; k < nc; ++k) {
+      const double un = cd_sh[k] - us * un_sh[k];
+      un_sh[k] = un;
+      b2 = fma(un, un, b2);
+    }
+    const double beta = sqrt(b2);
+    bsh[0] = beta;
+    bsh[1] = beta > 0.0 ? 1.0 / beta : 1.0;
+    bsh[2] = beta > 0.0 ? 1.0 : 0.0;
+    if (blockIdx.x == 0) {
+      st->pb_beta = beta;
+      st->pb_ib = bsh[1];
+      st->pb_pos = beta > 0.0;
+    }
+  }
+  __syncthreads();
+  if (blockIdx.x == 0 && threadIdx.x < nc) uc_tmp[threadIdx.x] = un_sh[threadIdx.x];
+  const double beta = bsh[0], ib = bsh[1];
+  if (bsh[2] == 0.0) return;  // beta == 0: v is left unchanged (P&S step b skipped)
+  double a2 = 0.0;
+  const int64_t na = 5 * S.n_stars;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < na; c += stride) {
+    double z = zA[c];
+    if (c < 5 * S.n_cs)
+      for (int64_t e = S.cs_ptr[c]; e < S.cs_ptr[c + 1]; ++e) z += S.cval[S.cs_e[e]] * un_sh[S.cs_k[e]];
+    const double vn = z * ib - beta * v[c];
+    v[c] = vn;
+    a2 = fma(vn, vn, a2);
+  }
+  double* vsh = v + S.A0;
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < S.n_sh; c += stride) {
+    double z = zsh[c];
+    if (c >= S.scs_lo && c < S.scs_hi) {
+      const int64_t q = c - S.scs_lo;
+      for (int64_t e = S.scs_ptr[q]; e < S.scs_ptr[q + 1]; ++e) z += S.cval[S.scs_e[e]] * un_sh[S.scs_k[e]];
+    }
+    const double vn = z * ib - beta * vsh[c];
+    vsh[c] = vn;
+    zsh[c] = 0.0;
+    a2 = fma(vn, vn, a2);
+  }
+  a2 = block_sum<kRedThreads>(a2);
+  if (threadIdx.x == 0) part_a2[blockIdx.x] = a2;
+}
+
+cudaError_t launch_post(const SysView& S, double* v, const double* zA, double* zsh, const double* part_rows,
+                        int64_t n_part, const double* cpart, const double* uc, double* uc_tmp, double* part_a2,
+                        int nblk, DevState* st, cudaStream_t s) {
+  k_post<<<nblk, kRedThreads, 0, s>>>(S, v, zA, zsh, part_rows, n_part, cpart, uc, uc_tmp, part_a2, st);
+  return cudaGetLastError();
+}
+
 // ------------------------------------------------------------------------------------------------ scale rows (O-PREC)
 __global__ void __launch_bounds__(kThreads, 1)
     k_scale_rows(SysView S, double* __restrict__ vals, const double* __restrict__ D) {
@@ -995,30 +1110,41 @@ __global__ void __launch_bounds__(kRedThreads)
     k_scalar(DevState* __restrict__ st, const double* __restrict__ part_astro, int64_t n_pa,
              const double* __restrict__ part_sh, int64_t n_ps, const double* __restrict__ part_wa, int64_t n_pwa,
              const double* __restrict__ part_ws, int64_t n_pws, const double* __restrict__ ar2_alpha2,
-             const double* __restrict__ ar1_wa, int init, int32_t* __restrict__ host_flag) {
+             const double* __restrict__ ar1_wa, int init, int32_t* __restrict__ host_flag,
+             const double* __restrict__ post_uc, double* __restrict__ uc, double* __restrict__ ucn, int nc) {
   if (!init && st->halted) {
     if (threadIdx.x == 0) st->col_enable = 0;
     return;
   }
-  const int bp = st->beta_pos;
+  // post_uc != nullptr: single-rank fused mode; beta and the new constraint u_hat come from k_post's hand-over
+  const int bp = post_uc ? st->pb_pos : st->beta_pos;
+  if (post_uc && threadIdx.x < nc) {
+    uc[threadIdx.x] = post_uc[threadIdx.x];
+    ucn[threadIdx.x] = post_uc[threadIdx.x] * st->pb_ib;
+  }
   // alpha^2 = ||v'||^2: astro part (per-warp partials of aprod2, or the allreduced value on several ranks)
   // + shared part (replicated, counted once).  ||w||^2 likewise (for ddnorm).
-  double a2 = 0.0;
-  if (bp) {
-    a2 = ar2_alpha2 ? 0.0 : ordered_sum<kRedThreads>(part_astro, n_pa);
-    a2 += ordered_sum<kRedThreads>(part_sh, n_ps);
-  }
-  double w2 = 0.0;
-  if (!init) {
-    w2 = ar1_wa ? 0.0 : ordered_sum<kRedThreads>(part_wa, n_pwa);
-    w2 += ordered_sum<kRedThreads>(part_ws, n_pws);
-  }
+  double sums[4] = {0.0, 0.0, 0.0, 0.0};
+  ordered_sum4<kRedThreads>(part_astro, (bp && !ar2_alpha2) ? n_pa : 0, part_sh, bp ? n_ps : 0, part_wa,
+                            (!init && !ar1_wa) ? n_pwa : 0, part_ws, init ? 0 : n_pws, sums);
+  double a2 = sums[0] + sums[1];
+  double w2 = sums[2] + sums[3];
   if (threadIdx.x != 0) return;
   if (bp && ar2_alpha2) a2 += *ar2_alpha2;
   if (!init && ar1_wa) w2 += *ar1_wa;
   DevState* const gst = st;
   DevState L = *gst;  // all loads issued together; computed on registers, written back once
   st = &L;
+  if (post_uc) {  // P&S step a/b bookkeeping for the new beta (was k_beta's job in the other modes)
+    const double beta = L.pb_beta;
+    if (L.pb_pos) {
+      const double a = L.alpha, d = L.damp;
+      L.anorm = sqrt(L.anorm * L.anorm + a * a + beta * beta + d * d);
+    }
+    L.beta = beta;
+    L.inv_beta = L.pb_ib;
+    L.beta_pos = L.pb_pos;
+  }
   const double eps = 0x1p-52;
   if (init) {
     const double alpha = bp ? sqrt(a2) : 0.0;
@@ -1355,9 +1481,9 @@ cudaError_t launch_add_shared(double* xsh, double* zsh, int64_t n, int mode, cud
 cudaError_t launch_scalar(DevState* st, const double* part_astro, int64_t n_pa, const double* part_sh,
                           int64_t n_ps, const double* part_wa, int64_t n_pwa, const double* part_ws, int64_t n_pws,
                           const double* ar2_alpha2, const double* ar1_wa, int init, int32_t* host_flag,
-                          cudaStream_t s) {
+                          cudaStream_t s, const double* post_uc, double* uc, double* ucn, int nc) {
   k_scalar<<<1, kRedThreads, 0, s>>>(st, part_astro, n_pa, part_sh, n_ps, part_wa, n_pwa, part_ws, n_pws,
-                                     ar2_alpha2, ar1_wa, init, host_flag);
+                                     ar2_alpha2, ar1_wa, init, host_flag, post_uc, uc, ucn, nc);
   return cudaGetLastError();
 }
 cudaError_t launch_colupdate(double* v, double* w, double* x, double* var, int64_t n, int64_t A0, double* part_wa,
