@@ -253,8 +253,8 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   if (ev) cudaEventRecord(ev[1], s);
   if (fused && !multi) {  // 4 launches: fused rows, post (beta + v' everywhere), scalar, column update
     if (ev) cudaEventRecord(ev[2], s);
-    CKL(h, launch_post(S, h->v, h->zA, h->zsh, h->part_rows, h->W, h->cpart, h->uc, h->uc_tmp, h->part_va, kG3,
-                       h->st, s), "post");
+    CKL(h, launch_post(S, h->v, h->zA, h->zsh, h->part_rows, h->grid, h->cpart, h->uc, h->uc_tmp, h->part_va,
+                       kG3, h->st, s), "post");
     if (ev) cudaEventRecord(ev[3], s);
     CKL(h, launch_scalar(h->st, h->part_va, kG3, nullptr, 0, h->part_wa, kG3, h->part_ws, kG3, nullptr, nullptr, 0,
                          h->hflag_dev, s, h->uc_tmp, h->uc, h->ucn, (int)h->n_constr), "scalar");
@@ -262,14 +262,15 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
         "colupdate");
     return LSQR_OK;
   }
+  const int64_t n_b2 = fused ? h->grid : h->W;  // k_fused publishes one beta^2 partial per CTA
   if (!multi) {
-    CKL(h, launch_beta(0, S, h->part_rows, h->W, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta");
+    CKL(h, launch_beta(0, S, h->part_rows, n_b2, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta");
   } else {
-    CKL(h, launch_beta(1, S, h->part_rows, h->W, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta1");
+    CKL(h, launch_beta(1, S, h->part_rows, n_b2, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta1");
     // AR1 payload: [constraint dots | beta^2 local | ||w_astro||^2 local]
     CKL(h, launch_sum_to(h->part_wa, kG3, h->ar1 + h->n_constr + 1, s), "wsum");
     CKR(allreduce(h, h->ar1, h->n_constr + 2));
-    CKL(h, launch_beta(2, S, h->part_rows, h->W, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta2");
+    CKL(h, launch_beta(2, S, h->part_rows, n_b2, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta2");
   }
   if (ev) cudaEventRecord(ev[2], s);
   const double* a2part;

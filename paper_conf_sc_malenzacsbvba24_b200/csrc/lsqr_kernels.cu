@@ -6,6 +6,7 @@
 // t=5 {astro 4, instr 4, instr 5, global}[j].  Each of the 6 loads of a warp instruction reads 8 rows x 32
 // contiguous bytes, so every fetched byte of A is used; the 4 lanes of a row hit 4 consecutive attitude columns,
 // which makes the attitude gathers (aprod1) and REDs (aprod2) sector-coalesced.
+#include <cstdlib>
 #include <type_traits>
 
 #include "lsqr_internal.cuh"
@@ -239,6 +240,12 @@ struct RingT {
   __device__ __forceinline__ const unsigned char* wait() const {
     mbar_wait(bar + 8 * slot, phase);
     return base + slot * kStage;
+  }
+  // wait for the stage AFTER the current one (software pipelining across stages)
+  __device__ __forceinline__ const unsigned char* wait_next() const {
+    const int s2 = slot + 1 == STAGES ? 0 : slot + 1;
+    mbar_wait(bar + 8 * s2, phase ^ (s2 == 0 ? 1u : 0u));
+    return base + s2 * kStage;
   }
 };
 using Ring = RingT<kRows, kStages>;
@@ -640,9 +647,9 @@ __global__ void __launch_bounds__(kThreads, 1)
 constexpr int kFRows = 8, kFStages = 4;
 using FRing = RingT<kFRows, kFStages>;
 constexpr int kSmemMaxBytes = 232448;  // 227 KB opt-in per CTA on sm_100
-constexpr int kFusedInstrMax = (kSmemMaxBytes - FRing::kBytes - FRing::kBars) / 16 - 2;
+constexpr int kFusedInstrMax = (kSmemMaxBytes - FRing::kBytes - FRing::kBars - 1024) / 16 - 2;  // 1 KB static
 
-template <bool SMEM_INSTR>
+template <bool SMEM_INSTR, int DIAG = 0>
 __global__ void __launch_bounds__(kThreads, 1)
     k_fused(SysView S, const double* __restrict__ x, double* __restrict__ u, double* __restrict__ zA,
             double* __restrict__ zsh, double* __restrict__ part, double* __restrict__ cpart,
@@ -720,46 +727,60 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   // one 8-row group: gathers, row dot, u_hat update, contributions.  CHECK: tail / star-boundary path with
   // per-lane validity and per-lane star; otherwise every lane's row is valid and in star cs.
-  auto group = [&](const unsigned char* stg, int g0, double uold, auto check_tag) {
+  // gathers of one 8-row group (attitude from L2, instrumental from shared memory), issued one group ahead of
+  // their use so their latency overlaps the previous group's arithmetic and scatters
+  struct Pre {
+    double g1, g2, g3, g4, g5;
+    int k0;
+    uint32_t i4, i5;
+  };
+  auto prefetch = [&](const unsigned char* stg, int g0) {
+    Pre P;
+    const bool valid = g0 + r < nrows;
+    const int4 q = *reinterpret_cast<const int4*>(stg + kFRows * kSlots * 8 + r * 16);
+    IdxRec rec;
+    rec.k0 = valid ? q.x : 0;
+    rec.ic01 = valid ? (uint32_t)q.y : 0u;
+    rec.ic23 = valid ? (uint32_t)q.z : 0u;
+    rec.ic45 = valid ? (uint32_t)q.w : 0u;
+    P.k0 = rec.k0;
+    P.i4 = ic4_of(rec, j);
+    P.i5 = (j == 3) ? (uint32_t)nsl : ic5_of(rec, j);
+    P.g1 = (DIAG & 4) ? 0.5 : __ldg(xatt0 + P.k0);
+    P.g2 = (DIAG & 4) ? 0.5 : __ldg(xatt1 + P.k0);
+    P.g3 = (DIAG & 4) ? 0.5 : __ldg(xatt2 + P.k0);
+    if (SMEM_INSTR) {
+      P.g4 = (DIAG & 8) ? 0.5 : sh_x[P.i4];
+      P.g5 = (DIAG & 8) ? 0.5 : sh_x[P.i5];
+    } else {
+      P.i5 = ic5_of(rec, j);
+      P.g4 = __ldg(xins_g + P.i4);
+      P.g5 = (j == 3) ? vglob_g : __ldg(xins_g + P.i5);
+    }
+    return P;
+  };
+
+  // one 8-row group: row dot, u_hat update, contributions.  CHECK: tail / star-boundary path with per-lane
+  // validity and per-lane star; otherwise every lane's row is valid and in star cs.
+  auto group = [&](const double (&v)[6], const Pre& P, int g0, double uold, auto check_tag) {
     constexpr bool CHECK = decltype(check_tag)::value;
     const int rel = g0 + r;
     const bool valid = !CHECK || rel < nrows;
-    double v[6];
-    IdxRec rec;
-    stage_row<kFRows>(stg, r, j, v, rec);
     double xj = cj, x4 = c4;
     int64_t my_s = cs;
-    if (CHECK) {
-      if (valid) {
-        int my_end = cs_end;
-        while (my_end <= rel) {
-          ++my_s;
-          my_end = (int)(S.star_ptr[my_s + 1] - r_lo);
-        }
-        if (my_s == cs + 1) { xj = nj; x4 = n4; }
-        else if (my_s != cs) { xj = __ldg(x + 5 * my_s + j); x4 = __ldg(x + 5 * my_s + 4); }
-      } else {
-        rec.k0 = 0; rec.ic01 = rec.ic23 = rec.ic45 = 0;
-#pragma unroll
-        for (int t = 0; t < 6; ++t) v[t] = 0.0;
+    if (CHECK && valid) {
+      int my_end = cs_end;
+      while (my_end <= rel) {
+        ++my_s;
+        my_end = (int)(S.star_ptr[my_s + 1] - r_lo);
       }
+      if (my_s == cs + 1) { xj = nj; x4 = n4; }
+      else if (my_s != cs) { xj = __ldg(x + 5 * my_s + j); x4 = __ldg(x + 5 * my_s + 4); }
     }
-    const int k0 = rec.k0;
-    const uint32_t i4 = ic4_of(rec, j);
-    const uint32_t i5 = (j == 3) ? (uint32_t)nsl : ic5_of(rec, j);
-    const double g1 = __ldg(xatt0 + k0), g2 = __ldg(xatt1 + k0), g3 = __ldg(xatt2 + k0);
-    double g4, g5;
-    if (SMEM_INSTR) {
-      g4 = sh_x[i4];
-      g5 = sh_x[i5];
-    } else {
-      g4 = __ldg(xins_g + i4);
-      g5 = (j == 3) ? vglob_g : __ldg(xins_g + ic5_of(rec, j));
-    }
-    g5 = (j == 0) ? x4 : g5;
-    double p = fma(v[1], g1, v[0] * xj);  // two short chains instead of one long one
-    double p2 = fma(v[4], g4, v[3] * g3);
-    p = fma(v[2], g2, p);
+    const double g5 = (j == 0) ? x4 : P.g5;
+    double p = fma(v[1], P.g1, v[0] * xj);  // two short chains instead of one long one
+    double p2 = fma(v[4], P.g4, v[3] * P.g3);
+    p = fma(v[2], P.g2, p);
     p2 = fma(v[5], g5, p2);
     p += p2;
     p += __shfl_xor_sync(0xffffffffu, p, 1);
@@ -770,19 +791,19 @@ __global__ void __launch_bounds__(kThreads, 1)
       b2 = fma(un, un, b2);
     }
     const double c1 = v[1] * un, c2 = v[2] * un, c3 = v[3] * un, c4v = v[4] * un, c5 = v[5] * un;
-    if (valid) {
-      atomicAdd(zatt0 + k0, c1);
-      atomicAdd(zatt1 + k0, c2);
-      atomicAdd(zatt2 + k0, c3);
+    if (valid && !(DIAG & 2)) {
+      atomicAdd(zatt0 + P.k0, c1);
+      atomicAdd(zatt1 + P.k0, c2);
+      atomicAdd(zatt2 + P.k0, c3);
     }
     if (SMEM_INSTR) {
-      double* ia[2] = {sh_z + i4, sh_z + i5};
+      double* ia[2] = {sh_z + P.i4, sh_z + P.i5};
       const double iv[2] = {c4v, c5};
-      const bool ion[2] = {valid, valid && t5_ins};
+      const bool ion[2] = {valid && !(DIAG & 1), valid && t5_ins && !(DIAG & 1)};
       smem_add_n<2>(ia, iv, ion);
     } else if (valid) {
-      atomicAdd(zins_g + i4, c4v);
-      if (t5_ins) atomicAdd(zins_g + ic5_of(rec, j), c5);
+      atomicAdd(zins_g + P.i4, c4v);
+      if (t5_ins) atomicAdd(zins_g + P.i5, c5);
     }
     gacc = fma(c5, m3, gacc);
     const double c0 = v[0] * un, c5a = c5 * m0;
@@ -802,36 +823,62 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int nst = (nrows + kFRows - 1) / kFRows;
   double uq0 = (r < nrows) ? __ldg(urow) : 0.0;            // u_hat of stage k (register queue, 2 deep)
   double uq1 = (kFRows + r < nrows) ? __ldg(urow + kFRows) : 0.0;
+  Pre Pc{};
+  if (nst > 0) Pc = prefetch(R.wait(), 0);
   for (int k = 0; k < nst; ++k) {
     const int g0 = k * kFRows;
     const double uold = uq0;
     uq0 = uq1;
     uq1 = (g0 + 2 * kFRows + r < nrows) ? __ldg(urow + g0 + 2 * kFRows) : 0.0;
     const unsigned char* stg = R.wait();
+    Pre Pn{};
+    if (k + 1 < nst) Pn = prefetch(R.wait_next(), g0 + kFRows);
+    double v[6];
+    {
+      const double2* rp = reinterpret_cast<const double2*>(stg + r * kSlots * 8 + 48 * j);
+#pragma unroll
+      for (int qq = 0; qq < 3; ++qq) {
+        const double2 d = rp[qq];
+        v[2 * qq] = d.x;
+        v[2 * qq + 1] = d.y;
+      }
+      if (g0 + r >= nrows) {
+#pragma unroll
+        for (int t = 0; t < 6; ++t) v[t] = 0.0;
+      }
+    }
+    R.release(lane);  // the stage's data is in registers: refill its slot now
     const bool fast = (g0 + kFRows <= nrows) && (cs_end >= g0 + kFRows);
     if (fast) {
-      group(stg, g0, uold, std::false_type{});
+      group(v, Pc, g0, uold, std::false_type{});
       while (cs < s_hi && cs_end <= g0 + kFRows) advance();
     } else {
-      group(stg, g0, uold, std::true_type{});
+      group(v, Pc, g0, uold, std::true_type{});
     }
-    R.release(lane);
+    Pc = Pn;
   }
   while (cs < s_hi) advance();  // empty trailing stars
   if (S.n_glob) {
     gacc = warp_sum(gacc);
     if (lane == 0 && gacc != 0.0) atomicAdd(zsh + S.n_att + S.n_instr, gacc);
   }
+  // beta^2: one partial per CTA (warps combined in a fixed order -> deterministic), so k_post re-sums few values
+  __shared__ double b2w[kWarpsPerCta];
   b2 = warp_sum(b2);
-  if (lane == 0) part[gw] = b2;
+  if (lane == 0) b2w[wid] = b2;
   for (int64_t c = gw; c < S.n_chunks; c += W) {  // constraint rows: owned-entry partial dots with v
     double acc = 0.0;
     for (int64_t e = S.ch_beg[c] + lane; e < S.ch_end[c]; e += 32) acc = fma(S.cval[e], __ldg(x + S.ccol[e]), acc);
     acc = warp_sum(acc);
     if (lane == 0) cpart[c] = acc;
   }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int q = 0; q < kWarpsPerCta; ++q) t += b2w[q];
+    part[blockIdx.x] = t;
+  }
   if (SMEM_INSTR) {
-    __syncthreads();
     for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
       const double vv = sh_z[S.ip.fwd(i)];
       if (vv != 0.0) atomicAdd(zsh + S.n_att + i, vv);
@@ -1448,24 +1495,43 @@ cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* p
   k_vshared<<<nblk, kRedThreads, 0, s>>>(S.n_sh, vsh, zsh, part, st, fused);
   return cudaGetLastError();
 }
-template <bool SM>
+template <bool SM, int DIAG>
 static cudaError_t fz(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh, double* part,
                       double* cpart, const DevState* st, cudaStream_t s) {
   const size_t smem = FRing::kBytes + FRing::kBars + (SM ? (2 * (size_t)S.ip.slots() + 4) * sizeof(double) : 0);
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_fused<SM>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemMaxBytes);
+  static size_t attr_set = 0;  // dynamic shared memory opted in so far (static shared memory counts separately)
+  if (smem > attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(k_fused<SM, DIAG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    attr_set = true;
+    attr_set = smem;
   }
-  k_fused<SM><<<grid, kThreads, smem, s>>>(S, x, u, zA, zsh, part, cpart, st);
+  k_fused<SM, DIAG><<<grid, kThreads, smem, s>>>(S, x, u, zA, zsh, part, cpart, st);
   return cudaGetLastError();
+}
+
+// LSQR_DIAG (debug experiments only; results are WRONG when set): bit 0 skips the instrumental CAS, bit 1 the
+// attitude REDs, bit 2 the attitude gathers, bit 3 the instrumental gathers.
+static int diag_mode() {
+  static int m = -1;
+  if (m < 0) {
+    const char* e = getenv("LSQR_DIAG");
+    m = e ? atoi(e) : 0;
+  }
+  return m;
 }
 
 cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh,
                          double* part, double* cpart, const DevState* st, cudaStream_t s) {
-  return S.ip.slots() <= kFusedInstrMax ? fz<true>(S, grid, x, u, zA, zsh, part, cpart, st, s)
-                                     : fz<false>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+  if (S.ip.slots() > kFusedInstrMax) return fz<false, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+  switch (diag_mode()) {
+    case 1: return fz<true, 1>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 2: return fz<true, 2>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 3: return fz<true, 3>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 4: return fz<true, 4>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 12: return fz<true, 12>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 15: return fz<true, 15>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    default: return fz<true, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+  }
 }
 
 cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const double* uc, double* zsh, double* part,
