@@ -250,8 +250,6 @@ struct RingT {
 };
 using Ring = RingT<kRows, kStages>;
 static_assert(Ring::kBytes == kRingBytes && Ring::kBars == kBarBytes, "ring geometry");
-constexpr int kA1Rows = 8, kA1Stages = 6;  // aprod1: one-group stages, software-pipelined gathers
-using A1Ring = RingT<kA1Rows, kA1Stages>;
 
 // row lr (0..kRows-1) of a stage: the lane's 6 values and the index record (16-B broadcast within the row group)
 template <int ROWS = kRows>
@@ -352,7 +350,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   extern __shared__ __align__(128) unsigned char dsm[];
   if (MODE == AP1_LSQR && st->halted) return;
   // the instrumental slice of x (<= 64 KB) is staged in shared memory: its gathers are random and L1-hostile
-  double* sh_x = reinterpret_cast<double*>(dsm + A1Ring::kBytes + A1Ring::kBars);
+  double* sh_x = reinterpret_cast<double*>(dsm + kRingBytes + kBarBytes);
   if (SMEM_INSTR) {
     for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_x[S.ip.fwd(i)] = x[S.I0 + i];
     __syncthreads();
@@ -362,7 +360,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const double uscale = MODE == AP1_LSQR ? st->u_scale : 0.0;
   const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
-  A1Ring R;
+  Ring R;
   R.setup(S, dsm, wid, lane, S.star_ptr[s_lo], S.star_ptr[s_hi]);
   R.prologue(lane);
   // loop-invariant per-lane gather bases (32-bit offsets inside the loop)
@@ -375,67 +373,57 @@ __global__ void __launch_bounds__(kThreads, 1)
   AstroCache ac;  // the lane's astrometric values of its current (and next) star live in registers
   ac.init(x, s_lo, s_hi, j);
   double b2 = 0.0;
-  const int nrows = (int)(R.r_hi - R.r_lo);
-  double* const yrow = y + R.r_lo + r;
-  // one 8-row group in registers: the lane's 6 values and its 6 gathered x values (issued one group ahead)
-  struct G {
-    double v[6], xv[6];
-  };
-  auto load_group = [&](const unsigned char* stg, int g0) {
-    G g;
-    const bool valid = g0 + r < nrows;
-    IdxRec rec;
-    stage_row<kA1Rows>(stg, r, j, g.v, rec);
-    if (valid && track_star(S, R.r_lo + g0 + r, s, bound)) ac.move_to(x, s, s_hi, j);
-    const int k0 = valid ? rec.k0 : 0;
-    g.xv[0] = ac.cj;
-    g.xv[1] = __ldg(xatt0 + k0);
-    g.xv[2] = __ldg(xatt1 + k0);
-    g.xv[3] = __ldg(xatt2 + k0);
-    const uint32_t i4 = valid ? ic4_of(rec, j) : 0u, i5 = valid ? ic5_of(rec, j) : 0u;
-    g.xv[4] = SMEM_INSTR ? xins[i4] : __ldg(xins + i4);
-    const double a_ins = SMEM_INSTR ? xins[i5] : __ldg(xins + i5);
-    g.xv[5] = j == 0 ? ac.c4 : (j == 3 ? vglob : a_ins);
-    if (!valid) {
+  double* yp = y + R.r_lo + r;  // this lane's row in the current group
+  double ynext[kGroups];
 #pragma unroll
-      for (int t = 0; t < 6; ++t) g.v[t] = 0.0;
+  for (int q = 0; q < kGroups; ++q) ynext[q] = (R.r_lo + q * 8 + r < R.r_hi) ? __ldg(yp + q * 8) : 0.0;
+  int64_t row0 = R.r_lo;
+  for (int64_t k = 0; k < R.nst; ++k, row0 += kRows, yp += kRows) {
+    double ycur[kGroups];
+#pragma unroll
+    for (int q = 0; q < kGroups; ++q) {  // prefetch next stage's y (u_hat)
+      ycur[q] = ynext[q];
+      ynext[q] = (row0 + kRows + q * 8 + r < R.r_hi) ? __ldg(yp + kRows + q * 8) : 0.0;
     }
-    return g;
-  };
-  const int nst = (nrows + kA1Rows - 1) / kA1Rows;
-  G gc{};
-  double yc = 0.0, yn = 0.0;
-  if (nst > 0) {
-    gc = load_group(R.wait(), 0);
+    const unsigned char* stg = R.wait();
+    double v[kGroups][6], xv[kGroups][6];
+    bool valid[kGroups];
+#pragma unroll
+    for (int q = 0; q < kGroups; ++q) {
+      const int64_t row = row0 + q * 8 + r;
+      valid[q] = row < R.r_hi;
+      IdxRec rec;
+      stage_row(stg, q * 8 + r, j, v[q], rec);
+      if (valid[q] && track_star(S, row, s, bound)) ac.move_to(x, s, s_hi, j);
+      // only the attitude values are gathered from global memory (L2) per row; instr from shared memory
+      const int k0 = valid[q] ? rec.k0 : 0;
+      xv[q][0] = ac.cj;
+      xv[q][1] = __ldg(xatt0 + k0);
+      xv[q][2] = __ldg(xatt1 + k0);
+      xv[q][3] = __ldg(xatt2 + k0);
+      const uint32_t i4 = valid[q] ? ic4_of(rec, j) : 0u, i5 = valid[q] ? ic5_of(rec, j) : 0u;
+      xv[q][4] = SMEM_INSTR ? xins[i4] : __ldg(xins + i4);
+      const double a_ins = SMEM_INSTR ? xins[i5] : __ldg(xins + i5);
+      xv[q][5] = j == 0 ? ac.c4 : (j == 3 ? vglob : a_ins);
+    }
     R.release(lane);
-    yc = (r < nrows) ? __ldg(yrow) : 0.0;
-  }
-  for (int k = 0; k < nst; ++k) {
-    const int g0 = k * kA1Rows;
-    G gn{};
-    if (k + 1 < nst) {  // next group: wait, load, issue its gathers, refill its slot
-      gn = load_group(R.wait(), g0 + kA1Rows);
-      R.release(lane);
-      yn = (g0 + kA1Rows + r < nrows) ? __ldg(yrow + g0 + kA1Rows) : 0.0;
-    }
-    double p = fma(gc.v[1], gc.xv[1], gc.v[0] * gc.xv[0]);
-    double p2 = fma(gc.v[4], gc.xv[4], gc.v[3] * gc.xv[3]);
-    p = fma(gc.v[2], gc.xv[2], p);
-    p2 = fma(gc.v[5], gc.xv[5], p2);
-    p += p2;
-    p += __shfl_xor_sync(0xffffffffu, p, 1);
-    p += __shfl_xor_sync(0xffffffffu, p, 2);
-    if (g0 + r < nrows && j == 0) {
-      if (MODE == AP1_LSQR) {
-        const double un = p - uscale * yc;
-        yrow[g0] = un;
-        b2 = fma(un, un, b2);
-      } else {
-        yrow[g0] = yc + p;
+#pragma unroll
+    for (int q = 0; q < kGroups; ++q) {
+      double p = 0.0;
+#pragma unroll
+      for (int t = 0; t < 6; ++t) p = fma(v[q][t], xv[q][t], p);
+      p += __shfl_xor_sync(0xffffffffu, p, 1);
+      p += __shfl_xor_sync(0xffffffffu, p, 2);
+      if (valid[q] && j == 0) {
+        if (MODE == AP1_LSQR) {
+          const double un = p - uscale * ycur[q];
+          yp[q * 8] = un;
+          b2 = fma(un, un, b2);
+        } else {
+          yp[q * 8] = ycur[q] + p;
+        }
       }
     }
-    gc = gn;
-    yc = yn;
   }
   if (MODE == AP1_LSQR) {
     b2 = warp_sum(b2);
@@ -1429,12 +1417,13 @@ cudaError_t launch_generate(const GenArgs& g, double* vals, IdxRec* idx, const i
 template <int MODE, bool SM>
 static cudaError_t ap1(const SysView& S, int grid, const double* x, double* y, double* part, double* cpart,
                        const DevState* st, cudaStream_t s) {
-  const size_t smem = A1Ring::kBytes + A1Ring::kBars + (SM ? (size_t)S.ip.slots() * sizeof(double) : 0);
-  static size_t attr_set = 0;
-  if (smem > attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_aprod1<MODE, SM>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  const size_t smem = kRingBytes + kBarBytes + (SM ? (size_t)S.ip.slots() * sizeof(double) : 0);
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(k_aprod1<MODE, SM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)(kRingBytes + kBarBytes + (SM ? (kInstrSmemMax + 64) * sizeof(double) : 0)));
     if (e != cudaSuccess) return e;
-    attr_set = smem;
+    attr_set = true;
   }
   k_aprod1<MODE, SM><<<grid, kThreads, smem, s>>>(S, x, y, part, cpart, st);
   return cudaGetLastError();
