@@ -241,10 +241,10 @@ struct RingT {
     mbar_wait(bar + 8 * slot, phase);
     return base + slot * kStage;
   }
-  // wait for the stage AFTER the current one (software pipelining across stages)
-  __device__ __forceinline__ const unsigned char* wait_next() const {
-    const int s2 = slot + 1 == STAGES ? 0 : slot + 1;
-    mbar_wait(bar + 8 * s2, phase ^ (s2 == 0 ? 1u : 0u));
+  // wait for the stage d positions after the current one (software pipelining across stages; d < STAGES)
+  __device__ __forceinline__ const unsigned char* wait_ahead(int d) const {
+    const int s2 = slot + d >= STAGES ? slot + d - STAGES : slot + d;
+    mbar_wait(bar + 8 * s2, phase ^ (slot + d >= STAGES ? 1u : 0u));
     return base + s2 * kStage;
   }
 };
@@ -644,7 +644,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 // algebraically the P&S step b (u = u_hat/beta).  Astro z goes to zA (scatter-free, per star), the shared slice to
 // z_sh exactly as in aprod2.  The ring is shallower (8-row stages) because v_instr (gathers) and z_instr
 // (accumulator) both live in shared memory.
-constexpr int kFRows = 8, kFStages = 4;
+constexpr int kFRows = 8, kFStages = 4, kFPre = 1;  // kFPre: gather prefetch distance in groups (2 measured slower: it shortens the TMA lead)
 using FRing = RingT<kFRows, kFStages>;
 constexpr int kSmemMaxBytes = 232448;  // 227 KB opt-in per CTA on sm_100
 constexpr int kFusedInstrMax = (kSmemMaxBytes - FRing::kBytes - FRing::kBars - 1024) / 16 - 2;  // 1 KB static
@@ -823,8 +823,10 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int nst = (nrows + kFRows - 1) / kFRows;
   double uq0 = (r < nrows) ? __ldg(urow) : 0.0;            // u_hat of stage k (register queue, 2 deep)
   double uq1 = (kFRows + r < nrows) ? __ldg(urow + kFRows) : 0.0;
-  Pre Pc{};
+  // gathers run kFPre groups ahead of their use (the stages they read are held in the ring until consumed)
+  Pre Pc{}, Pn1{};
   if (nst > 0) Pc = prefetch(R.wait(), 0);
+  if (kFPre > 1 && nst > 1) Pn1 = prefetch(R.wait_ahead(1), kFRows);
   for (int k = 0; k < nst; ++k) {
     const int g0 = k * kFRows;
     const double uold = uq0;
@@ -832,7 +834,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     uq1 = (g0 + 2 * kFRows + r < nrows) ? __ldg(urow + g0 + 2 * kFRows) : 0.0;
     const unsigned char* stg = R.wait();
     Pre Pn{};
-    if (k + 1 < nst) Pn = prefetch(R.wait_next(), g0 + kFRows);
+    if (k + kFPre < nst) Pn = prefetch(R.wait_ahead(kFPre), g0 + kFPre * kFRows);
     double v[6];
     {
       const double2* rp = reinterpret_cast<const double2*>(stg + r * kSlots * 8 + 48 * j);
@@ -855,7 +857,12 @@ __global__ void __launch_bounds__(kThreads, 1)
     } else {
       group(v, Pc, g0, uold, std::true_type{});
     }
-    Pc = Pn;
+    if (kFPre > 1) {
+      Pc = Pn1;
+      Pn1 = Pn;
+    } else {
+      Pc = Pn;
+    }
   }
   while (cs < s_hi) advance();  // empty trailing stars
   if (S.n_glob) {
