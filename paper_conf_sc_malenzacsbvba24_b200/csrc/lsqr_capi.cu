@@ -99,7 +99,7 @@ struct lsqr_ctx {
   double *part_wa = nullptr, *part_ws = nullptr, *part_g1 = nullptr, *ar1 = nullptr, *uc = nullptr,
          *ucn = nullptr, *crhs = nullptr, *tmp = nullptr, *tmax = nullptr;
   IdxRec* idx = nullptr;
-  int64_t *star_ptr = nullptr, *warp_star = nullptr;
+  int64_t *star_ptr = nullptr, *warp_star = nullptr, *warp_star_f = nullptr;
   DevState* st = nullptr;
   int32_t* hflag = nullptr;  // host-mapped
   int32_t* hflag_dev = nullptr;
@@ -498,15 +498,20 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   h->star_ptr_h.resize(h->n_loc_stars + 1);
   for (int64_t s = 0; s <= h->n_loc_stars; ++s) h->star_ptr_h[s] = rp[h->star_begin + s] - h->row_begin;
 
-  // warp partition: warp w starts at the first star whose rows begin at or after w*n_loc_rows/W
-  std::vector<int64_t> ws(h->W + 1);
-  for (int64_t w = 0; w < h->W; ++w) {
-    const int64_t target = (int64_t)((__int128)w * h->n_loc_rows / h->W);
-    ws[w] = std::lower_bound(h->star_ptr_h.begin(), h->star_ptr_h.end(), target) - h->star_ptr_h.begin();
-    if (ws[w] > h->n_loc_stars) ws[w] = h->n_loc_stars;
-  }
-  ws[0] = 0;
-  ws[h->W] = h->n_loc_stars;
+  // warp partitions: warp w starts at the first star whose rows begin at or after w*n_loc_rows/W (stars whole)
+  auto partition = [&](int64_t W) {
+    std::vector<int64_t> ws(W + 1);
+    for (int64_t w = 0; w < W; ++w) {
+      const int64_t target = (int64_t)((__int128)w * h->n_loc_rows / W);
+      ws[w] = std::lower_bound(h->star_ptr_h.begin(), h->star_ptr_h.end(), target) - h->star_ptr_h.begin();
+      if (ws[w] > h->n_loc_stars) ws[w] = h->n_loc_stars;
+    }
+    ws[0] = 0;
+    ws[W] = h->n_loc_stars;
+    return ws;
+  };
+  std::vector<int64_t> ws = partition(h->W);
+  std::vector<int64_t> wsf = partition((int64_t)h->grid * kFWarps);
 
   // ---- constraint ownership (O-SHARD): astro entries by the star's owner, shared entries by rank 0
   std::vector<double> cval;
@@ -586,6 +591,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   AL(h->u, h->n_loc_rows + 2);
   AL(h->star_ptr, h->n_loc_stars + 1);
   AL(h->warp_star, h->W + 1);
+  AL(h->warp_star_f, (int64_t)h->grid * kFWarps + 1);
   AL(h->v, h->n_loc_cols);
   AL(h->w, h->n_loc_cols);
   AL(h->x, h->n_loc_cols);
@@ -639,6 +645,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   };
   bool ok = up(h->star_ptr, h->star_ptr_h.data(), sizeof(int64_t) * h->star_ptr_h.size()) &&
             up(h->warp_star, ws.data(), sizeof(int64_t) * ws.size()) &&
+            up(h->warp_star_f, wsf.data(), sizeof(int64_t) * wsf.size()) &&
             up(d_cval, cval.data(), sizeof(double) * cval.size()) &&
             up(d_ccol, ccol.data(), sizeof(int64_t) * ccol.size()) &&
             up(d_chr, ch_row.data(), sizeof(int32_t) * ch_row.size()) &&
@@ -658,6 +665,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
 
   SysView& S = h->S;
   S.vals = h->vals; S.idx = h->idx; S.star_ptr = h->star_ptr; S.warp_star = h->warp_star;
+  S.warp_star_f = h->warp_star_f;
   S.n_rows = h->n_loc_rows; S.n_stars = h->n_loc_stars; S.n_axis = n_axis; S.n_att = n_att; S.n_instr = n_instr;
   S.n_sh = h->n_sh; S.n_cols = h->n_loc_cols; S.A0 = 5 * h->n_loc_stars; S.I0 = S.A0 + n_att;
   S.G0 = S.I0 + n_instr; S.n_glob = n_glob; S.n_constr = (int32_t)nc;

@@ -14,6 +14,8 @@ constexpr int kRows = 16;            // rows per TMA stage (two 8-row groups, 4 
 constexpr int kGroups = kRows / 8;
 constexpr int kStages = 3;           // ring depth per warp (kStages-1 stages in flight while computing)
 constexpr int kStageBytes = kRows * (kSlots * 8 + 16);                  // 3328 B: values + index records
+constexpr int kFWarps = 12;          // fused kernel: warps per CTA (its own warp partition, SysView::warp_star_f)
+constexpr int kFStages = 6;          // fused kernel: ring depth (8-row stages)
 constexpr int kRingBytes = kWarpsPerCta * kStages * kStageBytes;        // 159,744 B per CTA
 constexpr int kBarBytes = kWarpsPerCta * kStages * 8;                   // mbarriers
 constexpr int kRedThreads = 256;     // small reduction / vector kernels
@@ -90,6 +92,7 @@ struct SysView {
   const IdxRec* idx;        // [n_rows]
   const int64_t* star_ptr;  // [n_stars+1] local row offsets per local star
   const int64_t* warp_star; // [n_warps+1] star partition of the persistent warps (balanced by rows)
+  const int64_t* warp_star_f; // same for the fused kernel's warps (kFWarps per CTA)
   int64_t n_rows, n_stars, n_axis, n_att, n_instr, n_sh, n_cols, A0, I0, G0;
   int32_t n_glob, n_constr;
   // constraint entries OWNED by this rank (S:§8(c) O-SHARD), values scaled with A

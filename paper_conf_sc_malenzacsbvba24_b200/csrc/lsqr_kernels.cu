@@ -155,10 +155,19 @@ __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.
 __device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
 }
-__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-               "l"(src), "r"(bytes), "r"(bar)
-               : "memory");
+// A is streamed exactly once per pass: its TMA copies carry an L2 evict-first policy so they do not displace the
+// L2-resident shared-slice vectors (v_att/z_att: 24 MB at C4/C5) that the gathers and REDs hit.
+__device__ __forceinline__ uint64_t l2_evict_first_policy() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar, uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::
+          "r"(dst),
+      "l"(src), "r"(bytes), "r"(bar), "l"(pol)
+      : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
   asm volatile(
@@ -174,11 +183,11 @@ __device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
 
 // Per-warp ring state, templated on rows per stage and ring depth.  Stage counters advance incrementally (no
 // div/mod); lane 0 owns the issue pointers.
-template <int ROWS, int STAGES>
+template <int ROWS, int STAGES, int NW = kWarpsPerCta>
 struct RingT {
   static constexpr int kStage = ROWS * (kSlots * 8 + 16);
-  static constexpr int kBytes = kWarpsPerCta * STAGES * kStage;
-  static constexpr int kBars = kWarpsPerCta * STAGES * 8;
+  static constexpr int kBytes = NW * STAGES * kStage;
+  static constexpr int kBars = NW * STAGES * 8;
   const unsigned char* base;  // generic address of this warp's stage 0
   uint32_t ring, bar;         // shared addresses of stage 0 and mbarrier 0
   int64_t r_lo, r_hi, nst;    // row range and number of stages
@@ -189,6 +198,7 @@ struct RingT {
   const double* vsrc;
   const IdxRec* isrc;
   int64_t left;
+  uint64_t pol;               // L2 evict-first policy for the streamed rows
 
   __device__ __forceinline__ void setup(const SysView& S, unsigned char* dsm, int wid, int lane, int64_t lo,
                                         int64_t hi) {
@@ -205,6 +215,7 @@ struct RingT {
     vsrc = S.vals + lo * kSlots;
     isrc = S.idx + lo;
     left = hi - lo;
+    pol = l2_evict_first_policy();
     if (lane == 0) {
       for (int q = 0; q < STAGES; ++q) mbar_init(bar + 8 * q, 1);
       fence_mbar_init();
@@ -215,8 +226,8 @@ struct RingT {
     const uint32_t n = (uint32_t)(left < ROWS ? left : ROWS);
     const uint32_t b = bar + 8 * islot, dst = ring + islot * kStage;
     mbar_expect_tx(b, n * (kSlots * 8 + 16));
-    bulk_g2s(dst, vsrc, n * (kSlots * 8), b);
-    bulk_g2s(dst + ROWS * kSlots * 8, isrc, n * 16, b);
+    bulk_g2s(dst, vsrc, n * (kSlots * 8), b, pol);
+    bulk_g2s(dst + ROWS * kSlots * 8, isrc, n * 16, b, pol);
     vsrc += ROWS * kSlots;
     isrc += ROWS;
     left -= n;
@@ -644,13 +655,13 @@ __global__ void __launch_bounds__(kThreads, 1)
 // algebraically the P&S step b (u = u_hat/beta).  Astro z goes to zA (scatter-free, per star), the shared slice to
 // z_sh exactly as in aprod2.  The ring is shallower (8-row stages) because v_instr (gathers) and z_instr
 // (accumulator) both live in shared memory.
-constexpr int kFRows = 8, kFStages = 4, kFPre = 1;  // kFPre: gather prefetch distance in groups (2 measured slower: it shortens the TMA lead)
-using FRing = RingT<kFRows, kFStages>;
+constexpr int kFRows = 8, kFPre = 1;  // kFPre: gather prefetch distance in groups (2 measured slower)
+using FRing = RingT<kFRows, kFStages, kFWarps>;
 constexpr int kSmemMaxBytes = 232448;  // 227 KB opt-in per CTA on sm_100
 constexpr int kFusedInstrMax = (kSmemMaxBytes - FRing::kBytes - FRing::kBars - 1024) / 16 - 2;  // 1 KB static
 
 template <bool SMEM_INSTR, int DIAG = 0>
-__global__ void __launch_bounds__(kThreads, 1)
+__global__ void __launch_bounds__(kFWarps * 32, 1)
     k_fused(SysView S, const double* __restrict__ x, double* __restrict__ u, double* __restrict__ zA,
             double* __restrict__ zsh, double* __restrict__ part, double* __restrict__ cpart,
             const DevState* __restrict__ st) {
@@ -674,7 +685,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const double uscale = st->u_scale;
-  const int64_t s_lo = S.warp_star[gw], s_hi = S.warp_star[gw + 1];
+  const int64_t s_lo = S.warp_star_f[gw], s_hi = S.warp_star_f[gw + 1];
   const int64_t r_lo = S.star_ptr[s_lo];
   const int nrows = (int)(S.star_ptr[s_hi] - r_lo);  // rows of this warp (< 2^31)
   FRing R;
@@ -787,7 +798,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     p += __shfl_xor_sync(0xffffffffu, p, 2);
     const double un = valid ? p - uscale * uold : 0.0;  // identical in the row's 4 lanes
     if (j == 0 && valid) {
-      urow[g0] = un;
+      __stcs(urow + g0, un);
       b2 = fma(un, un, b2);
     }
     const double c1 = v[1] * un, c2 = v[2] * un, c3 = v[3] * un, c4v = v[4] * un, c5 = v[5] * un;
@@ -821,8 +832,8 @@ __global__ void __launch_bounds__(kThreads, 1)
   };
 
   const int nst = (nrows + kFRows - 1) / kFRows;
-  double uq0 = (r < nrows) ? __ldg(urow) : 0.0;            // u_hat of stage k (register queue, 2 deep)
-  double uq1 = (kFRows + r < nrows) ? __ldg(urow + kFRows) : 0.0;
+  double uq0 = (r < nrows) ? __ldcs(urow) : 0.0;           // u_hat of stage k (register queue, 2 deep;
+  double uq1 = (kFRows + r < nrows) ? __ldcs(urow + kFRows) : 0.0;  // streaming loads: evict-first in L2)
   // gathers run kFPre groups ahead of their use (the stages they read are held in the ring until consumed)
   Pre Pc{}, Pn1{};
   if (nst > 0) Pc = prefetch(R.wait(), 0);
@@ -831,7 +842,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int g0 = k * kFRows;
     const double uold = uq0;
     uq0 = uq1;
-    uq1 = (g0 + 2 * kFRows + r < nrows) ? __ldg(urow + g0 + 2 * kFRows) : 0.0;
+    uq1 = (g0 + 2 * kFRows + r < nrows) ? __ldcs(urow + g0 + 2 * kFRows) : 0.0;
     const unsigned char* stg = R.wait();
     Pre Pn{};
     if (k + kFPre < nst) Pn = prefetch(R.wait_ahead(kFPre), g0 + kFPre * kFRows);
@@ -870,7 +881,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     if (lane == 0 && gacc != 0.0) atomicAdd(zsh + S.n_att + S.n_instr, gacc);
   }
   // beta^2: one partial per CTA (warps combined in a fixed order -> deterministic), so k_post re-sums few values
-  __shared__ double b2w[kWarpsPerCta];
+  __shared__ double b2w[kFWarps];
   b2 = warp_sum(b2);
   if (lane == 0) b2w[wid] = b2;
   for (int64_t c = gw; c < S.n_chunks; c += W) {  // constraint rows: owned-entry partial dots with v
@@ -882,7 +893,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   __syncthreads();
   if (threadIdx.x == 0) {
     double t = 0.0;
-    for (int q = 0; q < kWarpsPerCta; ++q) t += b2w[q];
+    for (int q = 0; q < kFWarps; ++q) t += b2w[q];
     part[blockIdx.x] = t;
   }
   if (SMEM_INSTR) {
@@ -1512,7 +1523,7 @@ static cudaError_t fz(const SysView& S, int grid, const double* x, double* u, do
     if (e != cudaSuccess) return e;
     attr_set = smem;
   }
-  k_fused<SM, DIAG><<<grid, kThreads, smem, s>>>(S, x, u, zA, zsh, part, cpart, st);
+  k_fused<SM, DIAG><<<grid, kFWarps * 32, smem, s>>>(S, x, u, zA, zsh, part, cpart, st);
   return cudaGetLastError();
 }
 
