@@ -1527,8 +1527,10 @@ static cudaError_t fz(const SysView& S, int grid, const double* x, double* u, do
   return cudaGetLastError();
 }
 
-// LSQR_DIAG (debug experiments only; results are WRONG when set): bit 0 skips the instrumental CAS, bit 1 the
-// attitude REDs, bit 2 the attitude gathers, bit 3 the instrumental gathers.
+// Build-time experiment switch (not in the product build): compile with -DLSQR_DIAG_EXPERIMENTS to let the env var
+// LSQR_DIAG select kernel variants that skip work (results are WRONG): bit 0 the instrumental CAS, bit 1 the
+// attitude REDs, bit 2 the attitude gathers, bit 3 the instrumental gathers.  Used for DESIGN.md §7's time breakdown.
+#ifdef LSQR_DIAG_EXPERIMENTS
 static int diag_mode() {
   static int m = -1;
   if (m < 0) {
@@ -1537,19 +1539,21 @@ static int diag_mode() {
   }
   return m;
 }
+#endif
 
 cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh,
                          double* part, double* cpart, const DevState* st, cudaStream_t s) {
   if (S.ip.slots() > kFusedInstrMax) return fz<false, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+#ifdef LSQR_DIAG_EXPERIMENTS
   switch (diag_mode()) {
     case 1: return fz<true, 1>(S, grid, x, u, zA, zsh, part, cpart, st, s);
     case 2: return fz<true, 2>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 3: return fz<true, 3>(S, grid, x, u, zA, zsh, part, cpart, st, s);
     case 4: return fz<true, 4>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 12: return fz<true, 12>(S, grid, x, u, zA, zsh, part, cpart, st, s);
     case 15: return fz<true, 15>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    default: return fz<true, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    default: break;
   }
+#endif
+  return fz<true, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
 }
 
 cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const double* uc, double* zsh, double* part,

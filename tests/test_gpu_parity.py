@@ -367,3 +367,53 @@ def test_set_system_roundtrip_and_validation(avu):
     out = s.solve(itn_limit=50, atol=0, btol=0, conlim=0, fixed_count=True)
     assert out["itn"] == 50
     s.close()
+
+
+@pytest.mark.parametrize("case", ["instr_global", "empty_stars", "noglob"])
+def test_lsqr_fused_edge_cases(avu, case):
+    """Fused and two-pass iterations on the paths the default configs do not exercise: the instrumental slice too
+    large for shared memory (global-memory gathers/REDs), stars with no observations, no global column."""
+    if case == "instr_global":
+        w = W.C1.replace(name="C1i", n_instr=24_000, n_obs=30_000)
+        counts = None
+    elif case == "empty_stars":
+        w = W.micro(n_stars=50, obs=12, n_ext=6, seed=17)
+        counts = oracle.star_counts(w)
+        counts[[3, 4, 20, 49]] = 0
+        counts[0] += w.n_obs - counts.sum()
+    else:
+        w = W.C1C.replace(name="C1ng", n_glob=0)
+        counts = None
+    S = oracle.System(w, generate=False)
+    if counts is not None:  # user-provided obs-per-star: rebuild the oracle system and upload it
+        S.counts = counts
+        S.row_ptr = oracle.row_ptr(counts)
+        w2 = w
+        import ctypes
+        L = oracle.lib()
+        n = int(counts.sum())
+        S.n_rows, S.row_begin, S.row_end, S.star_begin, S.star_end = n, 0, n, 0, w.n_stars
+        S.vals = np.zeros((n, 24)); S.mA = np.zeros(n, dtype=np.int64); S.mT = np.zeros(n, dtype=np.int64)
+        S.iC = np.zeros((n, 6), dtype=np.int64); S.b = np.zeros(n)
+        P = lambda a: a.ctypes.data_as(ctypes.c_void_p)
+        L.orc_generate(w.seed, w.n_stars, w.n_att, w.n_instr, w.n_glob, P(S.row_ptr), 0, w.n_stars, P(S.vals),
+                       P(S.mA), P(S.mT), P(S.iC))
+        L.orc_generate_b(w.seed, 0, 0.0, w.n_stars, w.n_att, w.n_instr, w.n_glob, P(S.row_ptr), 0, w.n_stars,
+                         P(S.vals), P(S.mA), P(S.mT), P(S.iC), P(np.zeros(1)), P(S.b))
+        S._mk_struct()
+    else:
+        S = oracle.System(w)
+    ro = oracle.solve_system(S, itn_limit=150, atol=0, btol=0, conlim=0, fixed_count=True)
+    for fused in (True, False):
+        if counts is None:
+            s = avu.Solver.synthetic(w)
+        else:
+            s = avu.Solver(w.n_stars, w.n_obs, w.n_att, w.n_instr, w.n_glob, obs_per_star=counts,
+                           constraints=(S.c_ptr, S.c_col, S.c_val))
+            s.set_system(S.vals, S.mA, S.mT, S.iC, S.b)
+        s.precondition()
+        out = s.solve(itn_limit=150, atol=0, btol=0, conlim=0, fixed_count=True, fused=fused)
+        s.close()
+        assert out["itn"] == 150
+        assert rel(out["x"], ro["x"]) <= 1e-9, (case, fused, rel(out["x"], ro["x"]))
+        assert abs(out["r1norm"] - ro["r1norm"]) <= 1e-9 * ro["r1norm"]
