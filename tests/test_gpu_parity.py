@@ -373,8 +373,8 @@ def test_set_system_roundtrip_and_validation(avu):
 def test_lsqr_fused_edge_cases(avu, case):
     """Fused and two-pass iterations on the paths the default configs do not exercise: the instrumental slice too
     large for shared memory (global-memory gathers/REDs), stars with no observations, no global column."""
-    if case == "instr_global":
-        w = W.C1.replace(name="C1i", n_instr=24_000, n_obs=30_000)
+    if case == "instr_global":  # 120k rows x 30.2k columns (overdetermined), instrumental slice 192 KB
+        w = W.C1.replace(name="C1i", n_instr=24_000, n_obs=120_000)
         counts = None
     elif case == "empty_stars":
         w = W.micro(n_stars=50, obs=12, n_ext=6, seed=17)
@@ -403,6 +403,7 @@ def test_lsqr_fused_edge_cases(avu, case):
         S._mk_struct()
     else:
         S = oracle.System(w)
+    host = {k: getattr(S, k).copy() for k in ("vals", "mA", "mT", "iC", "b")}  # solve_system scales S in place
     ro = oracle.solve_system(S, itn_limit=150, atol=0, btol=0, conlim=0, fixed_count=True)
     for fused in (True, False):
         if counts is None:
@@ -410,7 +411,7 @@ def test_lsqr_fused_edge_cases(avu, case):
         else:
             s = avu.Solver(w.n_stars, w.n_obs, w.n_att, w.n_instr, w.n_glob, obs_per_star=counts,
                            constraints=(S.c_ptr, S.c_col, S.c_val))
-            s.set_system(S.vals, S.mA, S.mT, S.iC, S.b)
+            s.set_system(host["vals"], host["mA"], host["mT"], host["iC"], host["b"])
         s.precondition()
         out = s.solve(itn_limit=150, atol=0, btol=0, conlim=0, fixed_count=True, fused=fused)
         s.close()
