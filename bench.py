@@ -198,20 +198,28 @@ def run_ours(args):
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = 0 if args.same_device else int(os.environ.get("LOCAL_RANK", "0"))
     n = world
     torch.cuda.set_device(local)
     multi = world > 1
+    use_nccl = args.comm == "nccl"
     if multi:
-        dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", local))
+        if use_nccl:
+            dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", local))
+        else:  # test mode: gloo + the library's host-callback communicator (ranks may share one GPU)
+            dist.init_process_group("gloo", rank=rank, world_size=world)
     base = W.CONFIGS[args.config]
     w = base.per_gpu(n) if n > 1 else base
     w = w.replace(name=base.name)
-    kw = {}
-    if multi:
+    def comm_kw():
+        """A FRESH ncclUniqueId per communicator (NCCL ids must not be reused), broadcast from rank 0."""
+        if not multi:
+            return {}
+        if not use_nccl:
+            return dict(comm="callback")
         obj = [avu.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
-        kw = dict(comm="nccl", nccl_id=obj[0])
+        return dict(comm="nccl", nccl_id=obj[0])
     K, Wm = args.steps, args.warmup
 
     def barrier():
@@ -222,15 +230,14 @@ def run_ours(args):
     def max_over_ranks(v):
         if not multi:
             return v
-        t = torch.tensor([v], dtype=torch.float64, device="cuda")
+        t = torch.tensor([v], dtype=torch.float64, device="cuda" if use_nccl else "cpu")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
     # ---------------- e2e through the public API with HOST buffers (set_system -> precondition -> solve -> x, se)
     e2e = None
     if args.e2e:
-        s0 = avu.Solver.synthetic(base.per_gpu(n).replace(name=base.name) if n > 1 else base, rank=rank,
-                                  nranks=world, **kw)
+        s0 = avu.Solver.synthetic(w, rank=rank, nranks=world, **comm_kw())
         g = s0.get_system()
         nloc_cols = s0.n_local_cols
         s0.close()
@@ -239,7 +246,7 @@ def run_ours(args):
         del g
         xo = torch.empty(nloc_cols, dtype=torch.float64).pin_memory()
         so = torch.empty(nloc_cols, dtype=torch.float64).pin_memory()
-        se = avu.Solver.synthetic(w, rank=rank, nranks=world, generate=False, **kw)
+        se = avu.Solver.synthetic(w, rank=rank, nranks=world, generate=False, **comm_kw())
         barrier()
         t0 = time.perf_counter()
         se.set_system_ptrs(pin["vals"].data_ptr(), pin["mA"].data_ptr(), pin["mT"].data_ptr(),
@@ -258,7 +265,7 @@ def run_ours(args):
         torch.cuda.synchronize()
 
     # ---------------- device-resident timing
-    s = avu.Solver.synthetic(w, rank=rank, nranks=world, **kw)
+    s = avu.Solver.synthetic(w, rank=rank, nranks=world, **comm_kw())
     t0 = time.perf_counter()
     s.precondition()
     s.init(itn_limit=K + Wm + 10, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=False, fused=args.fused)
@@ -337,6 +344,9 @@ def main():
     ap.add_argument("--fused", dest="fused", action="store_true", default=True,
                     help="fused single-pass iteration (SURVEY 8(f) NEXT-1; default)")
     ap.add_argument("--two-pass", dest="fused", action="store_false", help="two-pass iteration (aprod1 then aprod2)")
+    ap.add_argument("--comm", default="nccl", choices=["nccl", "gloo-callback"],
+                    help="multi-rank communicator (gloo-callback: test mode through the library's host callback)")
+    ap.add_argument("--same-device", action="store_true", help="test mode: every rank on cuda:0")
     args = ap.parse_args()
     if args.warmup < 3:
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)

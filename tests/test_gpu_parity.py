@@ -379,7 +379,7 @@ def test_lsqr_fused_edge_cases(avu, case):
     elif case == "empty_stars":
         w = W.micro(n_stars=50, obs=12, n_ext=6, seed=17)
         counts = oracle.star_counts(w)
-        counts[[3, 4, 20, 49]] = 0
+        counts[[10, 11, 30, 49]] = 0  # stars >= n_ext: their columns become exactly zero (D = 1, x = 0)
         counts[0] += w.n_obs - counts.sum()
     else:
         w = W.C1C.replace(name="C1ng", n_glob=0)
