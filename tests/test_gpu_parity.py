@@ -403,14 +403,15 @@ def test_lsqr_fused_edge_cases(avu, case):
         S._mk_struct()
     else:
         S = oracle.System(w)
-    host = {k: getattr(S, k).copy() for k in ("vals", "mA", "mT", "iC", "b")}  # solve_system scales S in place
+    # solve_system scales S (values AND constraint values) in place: keep unscaled copies for the GPU
+    host = {k: getattr(S, k).copy() for k in ("vals", "mA", "mT", "iC", "b", "c_ptr", "c_col", "c_val")}
     ro = oracle.solve_system(S, itn_limit=150, atol=0, btol=0, conlim=0, fixed_count=True)
     for fused in (True, False):
         if counts is None:
             s = avu.Solver.synthetic(w)
         else:
             s = avu.Solver(w.n_stars, w.n_obs, w.n_att, w.n_instr, w.n_glob, obs_per_star=counts,
-                           constraints=(S.c_ptr, S.c_col, S.c_val))
+                           constraints=(host["c_ptr"], host["c_col"], host["c_val"]))
             s.set_system(host["vals"], host["mA"], host["mT"], host["iC"], host["b"])
         s.precondition()
         out = s.solve(itn_limit=150, atol=0, btol=0, conlim=0, fixed_count=True, fused=fused)
