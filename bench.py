@@ -149,11 +149,14 @@ def _cpu_model():
 
 
 def config_block(w, n, args, extra=None):
-    c = {"workload": w.name, "n_stars_per_gpu": w.n_stars, "n_obs_per_gpu": w.n_obs, "n_att": w.n_att,
+    """w: the whole job's workload (weak scaling: n x the per-GPU shape)."""
+    a_gpu = w.a_bytes // n
+    c = {"workload": w.name, "n_stars_per_gpu": w.n_stars // n, "n_obs_per_gpu": w.n_obs // n, "n_att": w.n_att,
          "n_instr": w.n_instr, "n_glob": w.n_glob, "constraint_rows": w.n_constr, "obs_jitter_pct": w.jitter_pct,
-         "A_bytes_per_gpu": w.a_bytes, "preconditioned": True, "mode": "fixed-count (paper timing mode)",
-         "seed": w.seed, "parallelism": f"dp{n} (rows sharded by star)",
-         "l2": "no flush: A per GPU (%.2f GB) >> L2 (126 MB)" % (w.a_bytes / 1e9)}
+         "A_bytes_per_gpu": a_gpu, "total_rows": w.n_obs, "preconditioned": True,
+         "mode": "fixed-count (paper timing mode)", "seed": w.seed, "parallelism": f"dp{n} (rows sharded by star)",
+         "variant": "fused single pass" if getattr(args, "fused", False) else "two-pass",
+         "l2": "no flush: A per GPU (%.2f GB) >> L2 (126 MB)" % (a_gpu / 1e9)}
     if extra:
         c.update(extra)
     return c
@@ -302,7 +305,7 @@ def run_ours(args):
         "metric": METRIC, "value": ms_step * 1e-3, "unit": UNIT, "n_gpus": n, "steps": K, "warmup": Wm,
         "ms_per_step": ms_step, "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
         "data": "synthetic",
-        "config": config_block(w, n, args, {"total_rows": w.n_obs, "setup_s": round(t_setup, 3)}),
+        "config": config_block(w, n, args, {"setup_s": round(t_setup, 3)}),
         "roofline": {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak,
                      "peak_kind": f"{peak_kind} (MEASURED_PEAKS.json hbm_gbs, copy; burst)", "unit": "GB/s",
                      "frac": round(achieved / peak, 4), "traffic": load_traffic(w.name if n == 1 else None, kname),
