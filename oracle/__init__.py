@@ -93,8 +93,12 @@ def lib():
             L.orc_precond_D.argtypes = [vp, i64, vp]
             L.orc_scale.argtypes = [C.POINTER(SysStruct), vp]
             L.orc_lsqr.restype = C.c_int
-            L.orc_lsqr.argtypes = [i64, i64, vp, vp, vp, d, d, d, d, i64, i32, i32, vp, vp, vp,
+            L.orc_lsqr.argtypes = [i64, i64, vp, vp, vp, d, d, d, d, i64, i32, i32, i32, vp, vp, vp,
                                    C.POINTER(LsqrOut), vp, vp]
+            L.orc_eda_sum.restype = d
+            L.orc_eda_sum.argtypes = [vp, i64]
+            for f in (L.orc_aprod1_repro, L.orc_aprod2_repro):
+                f.argtypes = [C.POINTER(SysStruct), vp, vp]
             _lib = L
     return _lib
 
@@ -224,6 +228,16 @@ class System:
         assert x.size == self.n_cols and y.size == self.m_local
         lib().orc_aprod2(C.byref(self.S), _p(y), _p(x))
 
+    def aprod1_repro(self, x: np.ndarray, y: np.ndarray) -> None:
+        """NEXT-4: y += A x with exact (order-independent) row sums, docs/REPRO.md."""
+        assert x.size == self.n_cols and y.size == self.m_local
+        lib().orc_aprod1_repro(C.byref(self.S), _p(x), _p(y))
+
+    def aprod2_repro(self, y: np.ndarray, x: np.ndarray) -> None:
+        """NEXT-4: x += A^T y with exact (order-independent) column sums."""
+        assert x.size == self.n_cols and y.size == self.m_local
+        lib().orc_aprod2_repro(C.byref(self.S), _p(y), _p(x))
+
     def colnorms(self) -> np.ndarray:
         c = np.zeros(self.n_cols, dtype=np.float64)
         lib().orc_colnorms(C.byref(self.S), _p(c))
@@ -267,7 +281,7 @@ class System:
 
 # --------------------------------------------------------------------------------------------------- O-LSQR
 def lsqr(m: int, n: int, aprod, b: np.ndarray, damp=0.0, atol=1e-8, btol=1e-8, conlim=1e8, itn_limit=None,
-         fixed_count=False, reorth=False, trace=None, want_se=True, trace_vectors=True):
+         fixed_count=False, reorth=False, trace=None, want_se=True, trace_vectors=True, repro=False):
     """Paige-Saunders LSQR (O-LSQR).  ``aprod`` is either a System (C products) or a python callable
     aprod(mode, vin, vout) with mode 1: vout[m] += A vin[n], mode 2: vout[n] += A^T vin[m].
     ``trace(state_dict, u, v, w, x, var)`` is called after every iteration with COPIES of the vectors
@@ -282,7 +296,7 @@ def lsqr(m: int, n: int, aprod, b: np.ndarray, damp=0.0, atol=1e-8, btol=1e-8, c
     out = LsqrOut()
     keep = []
     if isinstance(aprod, System):
-        fn = C.cast(L.orc_sys_aprod, C.c_void_p)
+        fn = C.cast(L.orc_sys_aprod_repro if repro else L.orc_sys_aprod, C.c_void_p)
         ctx = C.cast(C.pointer(aprod.S), C.c_void_p)
     else:
         def _cb(mode, vin, vout, _ctx, _f=aprod):
@@ -310,7 +324,8 @@ def lsqr(m: int, n: int, aprod, b: np.ndarray, damp=0.0, atol=1e-8, btol=1e-8, c
         keep.append(tcb)
         tfn = C.cast(tcb, C.c_void_p)
     rc = L.orc_lsqr(m, n, fn, ctx, _p(b), damp, atol, btol, conlim, int(itn_limit), int(bool(fixed_count)),
-                    int(bool(reorth)), _p(x), _p(var), _p(se) if want_se else None, C.byref(out), tfn, None)
+                    int(bool(reorth)), int(bool(repro)), _p(x), _p(var), _p(se) if want_se else None, C.byref(out),
+                    tfn, None)
     if rc != 0:
         raise MemoryError("orc_lsqr allocation failed")
     res = out.as_dict()
@@ -318,13 +333,19 @@ def lsqr(m: int, n: int, aprod, b: np.ndarray, damp=0.0, atol=1e-8, btol=1e-8, c
     return res
 
 
+def eda_sum(a) -> float:
+    """NEXT-4 exact digit accumulator: order-independent sum of doubles (docs/REPRO.md)."""
+    a = np.ascontiguousarray(a, dtype=np.float64)
+    return lib().orc_eda_sum(_p(a), a.size)
+
+
 def solve_system(sysm: System, damp=0.0, atol=1e-8, btol=1e-8, conlim=1e8, itn_limit=100, fixed_count=True,
-                 precondition=True, trace=None):
+                 precondition=True, trace=None, repro=False):
     """Full single-rank oracle solve: O-PREC (if requested and not yet applied), O-LSQR, O-4 se, O-5 unscale."""
     if precondition and sysm.D is None:
         sysm.apply_precond()
     res = lsqr(sysm.m_local, sysm.n_cols, sysm, sysm.rhs(), damp=damp, atol=atol, btol=btol, conlim=conlim,
-               itn_limit=itn_limit, fixed_count=fixed_count, trace=trace)
+               itn_limit=itn_limit, fixed_count=fixed_count, trace=trace, repro=repro)
     if sysm.D is not None:
         res["x_scaled"] = res["x"].copy()
         res["x"] = sysm.D * res["x"]

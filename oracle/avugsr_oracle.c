@@ -251,6 +251,98 @@ void orc_aprod2(const orc_sys* S, const double* y, double* x) {
       if (orc_owned(S, S->c_col[e])) x[S->c_col[e]] = x[S->c_col[e]] + S->c_val[e] * y[S->n_rows + k];
 }
 
+
+/* ------------------------------------------------------------------------------------------------------------
+ * NEXT-4 bitwise-reproducible mode: exact digit accumulator (EDA), docs/REPRO.md.  Every reduction
+ * becomes an order-independent integer sum of exactly split FP64 terms, rounded once; both the oracle and the GPU
+ * implement the spec, so their iterates agree bit for bit.
+ * ---------------------------------------------------------------------------------------------------------- */
+#define ORC_EDA_L 5
+typedef struct { int64_t d[ORC_EDA_L]; } orc_eda;
+static const int orc_eda_B[ORC_EDA_L] = {-8, -48, -88, -128, -168}; /* digit d covers bits [B_d, B_d + 40) */
+
+void orc_eda_add(orc_eda* A, double c) {
+  uint64_t bits;
+  memcpy(&bits, &c, sizeof bits);
+  const int neg = (int)(bits >> 63);
+  const int ex = (int)((bits >> 52) & 0x7ff);
+  uint64_t M = bits & ((1ULL << 52) - 1);
+  int E;
+  if (ex == 0) {
+    E = -1074;
+  } else {
+    M |= 1ULL << 52;
+    E = ex - 1075;
+  }
+  if (M == 0) return;
+  for (int d = 0; d < ORC_EDA_L; ++d) {
+    const int sh = E - orc_eda_B[d];
+    uint64_t dig;
+    if (sh >= 40) dig = 0;
+    else if (sh >= 0) dig = (M << sh) & ((1ULL << 40) - 1);
+    else if (sh > -53) dig = (M >> (-sh)) & ((1ULL << 40) - 1);
+    else dig = 0;
+    A->d[d] += neg ? -(int64_t)dig : (int64_t)dig;
+  }
+}
+
+double orc_eda_round(const orc_eda* A) {
+  int64_t D[ORC_EDA_L];
+  for (int d = 0; d < ORC_EDA_L; ++d) D[d] = A->d[d];
+  for (int d = ORC_EDA_L - 1; d >= 1; --d) { /* carry-normalise: D_d in [0, 2^40) for d >= 1 */
+    const int64_t c = D[d] >> 40;            /* arithmetic shift = floor division (gcc) */
+    D[d] -= c * ((int64_t)1 << 40);
+    D[d - 1] += c;
+  }
+  double v = 0.0;
+  for (int d = 0; d < ORC_EDA_L; ++d) v = v + ldexp((double)D[d], orc_eda_B[d]);
+  return v;
+}
+
+/* sum of n doubles through the EDA (test hook) */
+double orc_eda_sum(const double* a, int64_t n) {
+  orc_eda A;
+  memset(&A, 0, sizeof A);
+  for (int64_t i = 0; i < n; ++i) orc_eda_add(&A, a[i]);
+  return orc_eda_round(&A);
+}
+
+/* repro aprod1: y_i <- y_i + round(EDA sum of a_is * x[col_is]) (rows), same for the owned constraint entries */
+void orc_aprod1_repro(const orc_sys* S, const double* x, double* y) {
+  for (int64_t i = 0; i < S->n_rows; ++i) {
+    orc_eda A;
+    memset(&A, 0, sizeof A);
+    for (int sl = 0; sl < ORC_SLOTS; ++sl) {
+      if (sl == 23 && S->n_glob == 0) continue;
+      orc_eda_add(&A, S->vals[i * ORC_SLOTS + sl] * x[orc_col(sl, i, S->mA, S->mT, S->iC, S->n_axis, S->G0)]);
+    }
+    y[i] = y[i] + orc_eda_round(&A);
+  }
+  for (int64_t k = 0; k < S->n_constr; ++k) {
+    orc_eda A;
+    memset(&A, 0, sizeof A);
+    for (int64_t e = S->c_ptr[k]; e < S->c_ptr[k + 1]; ++e)
+      if (orc_owned(S, S->c_col[e])) orc_eda_add(&A, S->c_val[e] * x[S->c_col[e]]);
+    y[S->n_rows + k] = y[S->n_rows + k] + orc_eda_round(&A);
+  }
+}
+
+/* repro aprod2: x_j <- x_j + round(EDA sum over rows and owned constraint entries of a_ij * y_i), every column */
+void orc_aprod2_repro(const orc_sys* S, const double* y, double* x) {
+  orc_eda* Z = (orc_eda*)calloc((size_t)S->n_cols, sizeof(orc_eda));
+  if (!Z) abort();
+  for (int64_t i = 0; i < S->n_rows; ++i)
+    for (int sl = 0; sl < ORC_SLOTS; ++sl) {
+      if (sl == 23 && S->n_glob == 0) continue;
+      orc_eda_add(&Z[orc_col(sl, i, S->mA, S->mT, S->iC, S->n_axis, S->G0)], S->vals[i * ORC_SLOTS + sl] * y[i]);
+    }
+  for (int64_t k = 0; k < S->n_constr; ++k)
+    for (int64_t e = S->c_ptr[k]; e < S->c_ptr[k + 1]; ++e)
+      if (orc_owned(S, S->c_col[e])) orc_eda_add(&Z[S->c_col[e]], S->c_val[e] * y[S->n_rows + k]);
+  for (int64_t j = 0; j < S->n_cols; ++j) x[j] = x[j] + orc_eda_round(&Z[j]);
+  free(Z);
+}
+
 /* ------------------------------------------------------------------------------------------------------------
  * O-PREC: the LSQR is "preconditioned" (§II-B); the paper gives no detail.  S:§8(c) Z2 reading:
  * Jacobi column scaling.  c_j = sum over all rows (constraints included) of a_ij^2; D_j = 1/sqrt(c_j) (1 if c_j = 0);
@@ -316,7 +408,20 @@ void orc_sys_aprod(int32_t mode, const double* in, double* out, void* ctx) {
   else orc_aprod2((const orc_sys*)ctx, in, out);
 }
 
+void orc_sys_aprod_repro(int32_t mode, const double* in, double* out, void* ctx) {
+  if (mode == 1) orc_aprod1_repro((const orc_sys*)ctx, in, out);
+  else orc_aprod2_repro((const orc_sys*)ctx, in, out);
+}
+
+static int orc_repro_mode = 0; /* set by orc_lsqr for the duration of a solve */
+
 static double orc_nrm2(const double* a, int64_t n) { /* plain sqrt(sum a^2) in order, S:§8(c) Z5 */
+  if (orc_repro_mode) { /* NEXT-4: order-independent exact sum of the rounded squares */
+    orc_eda A;
+    memset(&A, 0, sizeof A);
+    for (int64_t i = 0; i < n; ++i) orc_eda_add(&A, a[i] * a[i]);
+    return sqrt(orc_eda_round(&A));
+  }
   double s = 0.0;
   for (int64_t i = 0; i < n; ++i) s = s + a[i] * a[i];
   return sqrt(s);
@@ -346,8 +451,9 @@ static void orc_reorth(double* a, const double* Q, int64_t k, int64_t n) {
  * Returns 0, or -1 on allocation failure.
  */
 int orc_lsqr(int64_t m, int64_t n, orc_aprod_fn aprod, void* ctx, const double* b, double damp, double atol,
-             double btol, double conlim, int64_t itn_limit, int32_t fixed_count, int32_t reorth, double* x,
-             double* var, double* se, orc_lsqr_out* out, orc_trace_fn trace, void* trace_ctx) {
+             double btol, double conlim, int64_t itn_limit, int32_t fixed_count, int32_t reorth, int32_t repro,
+             double* x, double* var, double* se, orc_lsqr_out* out, orc_trace_fn trace, void* trace_ctx) {
+  orc_repro_mode = repro ? 1 : 0;
   const double eps = 0x1p-52;
   double* u = (double*)malloc(sizeof(double) * (size_t)(m > 0 ? m : 1));
   double* v = (double*)malloc(sizeof(double) * (size_t)(n > 0 ? n : 1));
@@ -433,13 +539,17 @@ int orc_lsqr(int64_t m, int64_t n, orc_aprod_fn aprod, void* ctx, const double* 
     tau = sn * phi;
     /* e. update x, w, var (old w used for var and x) */
     double t1 = phi / rho, t2 = -theta / rho, t3 = 1.0 / rho;
+    orc_eda DD;
+    memset(&DD, 0, sizeof DD);
     for (int64_t j = 0; j < n; ++j) {
       double dk = t3 * w[j];
       var[j] = var[j] + dk * dk;
-      ddnorm = ddnorm + dk * dk;
+      if (repro) orc_eda_add(&DD, dk * dk);
+      else ddnorm = ddnorm + dk * dk;
       x[j] = x[j] + t1 * w[j];
       w[j] = v[j] + t2 * w[j];
     }
+    if (repro) ddnorm = ddnorm + orc_eda_round(&DD); /* NEXT-4: order-independent */
     /* f. norm of x estimate */
     double delta = sn2 * rho, gambar = -cs2 * rho, rhs = phi - delta * z, zbar = rhs / gambar;
     xnorm = sqrt(xxnorm + zbar * zbar);
@@ -503,5 +613,6 @@ done:
   out->r1norm = r1norm; out->r2norm = r2norm; out->anorm = anorm; out->acond = acond; out->arnorm = arnorm;
   out->xnorm = xnorm; out->bnorm = bnorm;
   free(u); free(v); free(w); free(U); free(V);
+  orc_repro_mode = 0;
   return 0;
 }
