@@ -120,21 +120,22 @@ def load_traffic(workload, kernel):
 
 
 # ------------------------------------------------------------------------------------------------ cpu baseline
-def cpu_baseline(w, iters=3):
-    """The oracle (serial C, as it stands) on a bounded sample: the full system, `iters` LSQR iterations."""
+def cpu_baseline(w, iters=3, repro=False):
+    """The oracle (serial C, as it stands) on a bounded sample: the full system, `iters` LSQR iterations
+    (``repro``: the oracle's bitwise-reproducible mode, NEXT-4)."""
     import oracle
     t0 = time.perf_counter()
     S = oracle.System(w)
-    S.apply_precond()
+    S.apply_precond(repro=repro)
     t_setup = time.perf_counter() - t0
     stamps = []
     oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), atol=0, btol=0, conlim=0, itn_limit=iters + 1, fixed_count=True,
-                want_se=False, trace=lambda st: stamps.append(time.perf_counter()), trace_vectors=False)
+                want_se=False, trace=lambda st: stamps.append(time.perf_counter()), trace_vectors=False, repro=repro)
     per = [b - a for a, b in zip(stamps[:-1], stamps[1:])]
     v = float(np.median(per))
     return {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
             "sample": f"full {w.name} system ({w.n_obs} rows), {len(per)} timed LSQR iterations of the serial C "
-                      f"oracle after 1 untimed (setup {t_setup:.1f} s excluded)",
+                      f"oracle{' (repro mode)' if repro else ''} after 1 untimed (setup {t_setup:.1f} s excluded)",
             "cpu_model": _cpu_model(), "host_cores": os.cpu_count()}
 
 
@@ -148,6 +149,12 @@ def _cpu_model():
     return None
 
 
+def variant_name(args):
+    if getattr(args, "repro", False):
+        return "bitwise-reproducible (SURVEY 8(f) NEXT-4; exact digit reductions, verification mode)"
+    return "fused single pass" if getattr(args, "fused", False) else "two-pass"
+
+
 def config_block(w, n, args, extra=None):
     """w: the whole job's workload (weak scaling: n x the per-GPU shape)."""
     a_gpu = w.a_bytes // n
@@ -155,7 +162,7 @@ def config_block(w, n, args, extra=None):
          "n_instr": w.n_instr, "n_glob": w.n_glob, "constraint_rows": w.n_constr, "obs_jitter_pct": w.jitter_pct,
          "A_bytes_per_gpu": a_gpu, "total_rows": w.n_obs, "preconditioned": True,
          "mode": "fixed-count (paper timing mode)", "seed": w.seed, "parallelism": f"dp{n} (rows sharded by star)",
-         "variant": "fused single pass" if getattr(args, "fused", False) else "two-pass",
+         "variant": variant_name(args),
          "l2": "no flush: A per GPU (%.2f GB) >> L2 (126 MB)" % (a_gpu / 1e9)}
     if extra:
         c.update(extra)
@@ -250,6 +257,8 @@ def run_ours(args):
         xo = torch.empty(nloc_cols, dtype=torch.float64).pin_memory()
         so = torch.empty(nloc_cols, dtype=torch.float64).pin_memory()
         se = avu.Solver.synthetic(w, rank=rank, nranks=world, generate=False, **comm_kw())
+        if args.repro:
+            se.set_reproducible(True)
         barrier()
         t0 = time.perf_counter()
         se.set_system_ptrs(pin["vals"].data_ptr(), pin["mA"].data_ptr(), pin["mT"].data_ptr(),
@@ -269,6 +278,8 @@ def run_ours(args):
 
     # ---------------- device-resident timing
     s = avu.Solver.synthetic(w, rank=rank, nranks=world, **comm_kw())
+    if args.repro:
+        s.set_reproducible(True)
     t0 = time.perf_counter()
     s.precondition()
     s.init(itn_limit=K + Wm + 10, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=False, fused=args.fused)
@@ -287,7 +298,10 @@ def run_ours(args):
     peak, peak_kind = measured_peaks()
     ap1_b, ap2_b, it_b = algorithmic_bytes(w, s.n_local_rows, s.star_end - s.star_begin, s.n_shared,
                                            s.n_local_cols)
-    if args.fused:
+    if args.repro:
+        # NEXT-4: the whole iteration (7 launches) is one timed unit; the algorithmic bytes are the two-pass ones
+        kname, kb, kms = "repro iteration", it_b, t_ms / K
+    elif args.fused:
         # fused single pass (NEXT-1): A, indices, u_hat read once + u_hat written (224 B/row), v_astro read and
         # zA written (80 B/star), v_shared gathered and z_shared written once (16 B/column)
         n_st = s.star_end - s.star_begin
@@ -313,11 +327,13 @@ def run_ours(args):
         "iteration_roofline": {"algorithmic_bytes": it_b, "achieved_GBps": round(it_b / (ms_step * 1e-3) / 1e9, 1),
                                "frac": round(it_b / (ms_step * 1e-3) / 1e9 / peak, 4),
                                "aprod1_ms": round(ap1_ms, 4), "aprod2_ms": round(ap2_ms, 4),
-                               "aprod1_frac": round(ap1_b / (ap1_ms * 1e-3) / 1e9 / peak, 4),
+                               "aprod1_frac": (round(ap1_b / (ap1_ms * 1e-3) / 1e9 / peak, 4)
+                                               if not args.repro else None),
                                "aprod2_frac": (round(ap2_b / (ap2_ms * 1e-3) / 1e9 / peak, 4)
-                                               if not args.fused else None),
-                               "variant": "fused single pass (SURVEY 8(f) NEXT-1; bytes are its own 224 B/row)"
-                               if args.fused else "two-pass (SURVEY 8(a)); 440 B/row"},
+                                               if not (args.fused or args.repro) else None),
+                               "variant": variant_name(args) if args.repro else
+                               ("fused single pass (SURVEY 8(f) NEXT-1; bytes are its own 224 B/row)"
+                                if args.fused else "two-pass (SURVEY 8(a)); 440 B/row")},
         "gpu_launches": int(max_over_ranks(r["launches"])),
         "clocks": clk.summary(),
         "e2e": e2e,
@@ -325,7 +341,7 @@ def run_ours(args):
     }
     s.close()
     if rank == 0 and n == 1 and args.cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(base, iters=args.cpu_iters)
+        line["cpu_baseline"] = cpu_baseline(base, iters=args.cpu_iters, repro=args.repro)
     if rank == 0:
         print(json.dumps(line), flush=True)
     if multi:
@@ -347,12 +363,17 @@ def main():
     ap.add_argument("--fused", dest="fused", action="store_true", default=True,
                     help="fused single-pass iteration (SURVEY 8(f) NEXT-1; default)")
     ap.add_argument("--two-pass", dest="fused", action="store_false", help="two-pass iteration (aprod1 then aprod2)")
+    ap.add_argument("--repro", action="store_true",
+                    help="bitwise-reproducible mode (SURVEY 8(f) NEXT-4; single GPU; verification, not speed)")
     ap.add_argument("--comm", default="nccl", choices=["nccl", "gloo-callback"],
                     help="multi-rank communicator (gloo-callback: test mode through the library's host callback)")
     ap.add_argument("--same-device", action="store_true", help="test mode: every rank on cuda:0")
     args = ap.parse_args()
     if args.warmup < 3:
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)
+    if args.repro and int(os.environ.get("WORLD_SIZE", "1")) > 1:
+        print("--repro is single-GPU", file=sys.stderr)
+        return 2
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)

@@ -186,6 +186,16 @@ int lsqr_get_system(lsqr_t h, double* vals, int64_t* matrixIndexAstro, int64_t* 
 int lsqr_precondition(lsqr_t h);
 /* D (n_local_cols; host or device pointer).  All ones before lsqr_precondition. */
 int lsqr_get_precond(lsqr_t h, double* D);
+/* Bitwise-reproducible mode (docs/REPRO.md), on = 1 / off = 0; off by default.  When on,
+ * lsqr_precondition and the LSQR (lsqr_init / lsqr_iterate / lsqr_solve) compute every reduction -- the column sums
+ * of squares, the row dots of aprod1, the column sums of aprod2, ||u||, ||v|| and ddnorm -- as an exact,
+ * order-independent digit accumulation rounded once, and every other step as one IEEE operation without FMA
+ * contraction, in the order of Paige & Saunders' recurrence.  The iterates are then bit-identical run
+ * to run and to the CPU oracle's repro mode, independent of scheduling; lsqr_solve_params.fused is ignored and the
+ * iteration is several times slower than the default path (verification mode).  Single rank only
+ * (LSQR_EINVAL when nranks > 1).  Allocates 40 B per local column of digit storage (LSQR_ENOMEM).  Invalidates a
+ * previous lsqr_init; call before lsqr_precondition for a reproducible D. */
+int lsqr_set_reproducible(lsqr_t h, int32_t on);
 
 /* ---------------------------------------------------------------- products (hot path) */
 /* y += A^ x  (aprod1, Eq. (3)).  x: device [n_local_cols], y: device [n_local_rows + n_constr].  A^ = A D after

@@ -90,6 +90,7 @@ def lib():
             for f in (L.orc_aprod1, L.orc_aprod2):
                 f.argtypes = [C.POINTER(SysStruct), vp, vp]
             L.orc_colnorms.argtypes = [C.POINTER(SysStruct), vp]
+            L.orc_colnorms_repro.argtypes = [C.POINTER(SysStruct), vp]
             L.orc_precond_D.argtypes = [vp, i64, vp]
             L.orc_scale.argtypes = [C.POINTER(SysStruct), vp]
             L.orc_lsqr.restype = C.c_int
@@ -238,15 +239,15 @@ class System:
         assert x.size == self.n_cols and y.size == self.m_local
         lib().orc_aprod2_repro(C.byref(self.S), _p(y), _p(x))
 
-    def colnorms(self) -> np.ndarray:
+    def colnorms(self, repro: bool = False) -> np.ndarray:
         c = np.zeros(self.n_cols, dtype=np.float64)
-        lib().orc_colnorms(C.byref(self.S), _p(c))
+        (lib().orc_colnorms_repro if repro else lib().orc_colnorms)(C.byref(self.S), _p(c))
         return c
 
-    def apply_precond(self, c_total: np.ndarray | None = None) -> np.ndarray:
-        """O-PREC: D from the column sums of squares (given, e.g. summed over ranks, or computed here), then
-        scale the stored values in place."""
-        c = self.colnorms() if c_total is None else c_total
+    def apply_precond(self, c_total: np.ndarray | None = None, repro: bool = False) -> np.ndarray:
+        """O-PREC: D from the column sums of squares (given, e.g. summed over ranks, or computed here; ``repro``:
+        NEXT-4 exact sums), then scale the stored values in place."""
+        c = self.colnorms(repro) if c_total is None else c_total
         D = np.zeros(self.n_cols, dtype=np.float64)
         lib().orc_precond_D(_p(np.ascontiguousarray(c)), self.n_cols, _p(D))
         lib().orc_scale(C.byref(self.S), _p(D))
@@ -343,7 +344,7 @@ def solve_system(sysm: System, damp=0.0, atol=1e-8, btol=1e-8, conlim=1e8, itn_l
                  precondition=True, trace=None, repro=False):
     """Full single-rank oracle solve: O-PREC (if requested and not yet applied), O-LSQR, O-4 se, O-5 unscale."""
     if precondition and sysm.D is None:
-        sysm.apply_precond()
+        sysm.apply_precond(repro=repro)
     res = lsqr(sysm.m_local, sysm.n_cols, sysm, sysm.rhs(), damp=damp, atol=atol, btol=btol, conlim=conlim,
                itn_limit=itn_limit, fixed_count=fixed_count, trace=trace, repro=repro)
     if sysm.D is not None:

@@ -361,6 +361,24 @@ void orc_colnorms(const orc_sys* S, double* c) {
       if (orc_owned(S, S->c_col[e])) c[S->c_col[e]] = c[S->c_col[e]] + S->c_val[e] * S->c_val[e];
 }
 
+/* NEXT-4 (docs/REPRO.md): the same column sums of squares, each an order-independent EDA sum of the rounded
+ * squares a*a, rounded once; every c[j] is overwritten (no accumulation into a caller value). */
+void orc_colnorms_repro(const orc_sys* S, double* c) {
+  orc_eda* Z = (orc_eda*)calloc((size_t)(S->n_cols > 0 ? S->n_cols : 1), sizeof(orc_eda));
+  if (!Z) abort();
+  for (int64_t i = 0; i < S->n_rows; ++i)
+    for (int sl = 0; sl < ORC_SLOTS; ++sl) {
+      if (sl == 23 && S->n_glob == 0) continue;
+      double a = S->vals[i * ORC_SLOTS + sl];
+      orc_eda_add(&Z[orc_col(sl, i, S->mA, S->mT, S->iC, S->n_axis, S->G0)], a * a);
+    }
+  for (int64_t k = 0; k < S->n_constr; ++k)
+    for (int64_t e = S->c_ptr[k]; e < S->c_ptr[k + 1]; ++e)
+      if (orc_owned(S, S->c_col[e])) orc_eda_add(&Z[S->c_col[e]], S->c_val[e] * S->c_val[e]);
+  for (int64_t j = 0; j < S->n_cols; ++j) c[j] = orc_eda_round(&Z[j]);
+  free(Z);
+}
+
 void orc_precond_D(const double* c, int64_t n, double* D) {
   for (int64_t j = 0; j < n; ++j) D[j] = c[j] > 0.0 ? 1.0 / sqrt(c[j]) : 1.0;
 }

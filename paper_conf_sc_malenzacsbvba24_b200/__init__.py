@@ -243,6 +243,11 @@ class Solver:
         self._chk(_capi.lib().lsqr_get_precond(self._h, _p(D)))
         return D
 
+    def set_reproducible(self, on: bool = True):
+        """NEXT-4 bitwise-reproducible mode (docs/REPRO.md): exact order-independent reductions in precondition and
+        LSQR; call before precondition()."""
+        self._chk(_capi.lib().lsqr_set_reproducible(self._h, int(bool(on))))
+
     # ------------------------------------------------------------------ products
     def aprod1(self, x, y):
         """y += A^ x (device float64 tensors; y = [local rows | constraint rows])."""

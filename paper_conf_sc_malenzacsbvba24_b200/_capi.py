@@ -71,6 +71,7 @@ EXPORTS = {
     "lsqr_get_system": (C.c_int, [vp, vp, vp, vp, vp, vp]),
     "lsqr_precondition": (C.c_int, [vp]),
     "lsqr_get_precond": (C.c_int, [vp, vp]),
+    "lsqr_set_reproducible": (C.c_int, [vp, C.c_int32]),
     "lsqr_aprod1": (C.c_int, [vp, vp, vp]),
     "lsqr_aprod2": (C.c_int, [vp, vp, vp]),
     "lsqr_solve": (C.c_int, [vp, C.POINTER(SolveParams), C.POINTER(Result), vp, vp]),

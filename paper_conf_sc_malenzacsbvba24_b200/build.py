@@ -9,7 +9,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "liblsqr_avugsr.so")
-SOURCES = ["lsqr_kernels.cu", "lsqr_capi.cu"]
+SOURCES = ["lsqr_kernels.cu", "lsqr_repro.cu", "lsqr_capi.cu"]
 HEADERS = ["lsqr_internal.cuh", os.path.join(ROOT, "include", "lsqr_avugsr.h")]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

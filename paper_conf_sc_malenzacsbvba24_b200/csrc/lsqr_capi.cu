@@ -112,6 +112,9 @@ struct lsqr_ctx {
   lsqr_solve_params params{};
   cudaGraphExec_t gexec = nullptr;
   bool graph_ok = false;
+  // NEXT-4 bitwise-reproducible mode: digit buffers (lsqr_repro.cu)
+  bool repro = false;
+  long long *rzd = nullptr, *rsd = nullptr;
   std::string err;
 };
 
@@ -244,6 +247,13 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   cudaStream_t s = h->s;
   const bool multi = h->nranks > 1;
   const bool fused = h->params.fused != 0;
+  if (h->repro) {  // NEXT-4: 7 launches, all in lsqr_repro.cu
+    if (ev) cudaEventRecord(ev[0], s);
+    CKL(h, repro_iteration(S, h->u, h->uc, h->crhs, h->v, h->w, h->x, h->var, h->rzd, h->rsd, h->st, h->hflag_dev,
+                           0, s), "repro");
+    if (ev) for (int k = 1; k < 4; ++k) cudaEventRecord(ev[k], s);
+    return LSQR_OK;
+  }
   if (ev) cudaEventRecord(ev[0], s);
   if (fused) {  // NEXT-1: u_hat update and A^T u_hat in one read of A
     CKL(h, launch_fused(S, h->grid, h->v, h->u, h->zA, h->zsh, h->part_rows, h->cpart, h->st, s), "fused");
@@ -301,7 +311,7 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   return LSQR_OK;
 }
 
-int kernels_per_iteration(lsqr_t h) { return h->nranks > 1 ? 9 : (h->params.fused ? 4 : 6); }
+int kernels_per_iteration(lsqr_t h) { return h->repro ? 7 : (h->nranks > 1 ? 9 : (h->params.fused ? 4 : 6)); }
 
 int build_graph(lsqr_t h) {
   if (h->gexec) {
@@ -827,6 +837,15 @@ int lsqr_precondition(lsqr_t h) {
   if (h->preconditioned) return fail(h, LSQR_ESTATE, "already preconditioned");
   SysView& S = h->S;
   enter(h);
+  if (h->repro) {  // NEXT-4: exact column sums of squares
+    CKL(h, repro_colnorm_D(S, h->D, h->rzd, h->s), "colnorm_repro");
+    CKL(h, launch_scale_rows(S, h->grid, h->vals, h->D, h->s), "scale_rows");
+    CKL(h, launch_scale_constr(S, const_cast<double*>(S.cval), h->D, h->s), "scale_constr");
+    leave(h);
+    h->preconditioned = true;
+    h->initialized = false;
+    return LSQR_OK;
+  }
   // c_j = sum a_ij^2: astro columns straight into D, shared slice accumulated in zsh (+ AR), then D = 1/sqrt(c)
   CKL(h, launch_aprod2(AP2_COLNORM, S, h->grid, nullptr, nullptr, h->D, h->zsh, h->part_a2, h->st, h->rank == 0,
                        h->s), "colnorm");
@@ -848,6 +867,21 @@ int lsqr_get_precond(lsqr_t h, double* D) {
   CKC(h, cudaStreamSynchronize(h->s));
   CKC(h, cudaMemcpy(D, h->D, sizeof(double) * h->n_loc_cols, cudaMemcpyDefault));
   leave(h);
+  return LSQR_OK;
+}
+
+int lsqr_set_reproducible(lsqr_t h, int32_t on) {
+  GUARD(h);
+  if (on != 0 && on != 1) return LSQR_EINVAL;
+  if (on && h->nranks > 1) return fail(h, LSQR_EINVAL, "reproducible mode is single-rank");
+  if (on && !h->rzd) {
+    CKR(dalloc(h, &h->rzd, repro_digits_per_value() * h->n_loc_cols));
+    CKR(dalloc(h, &h->rsd, repro_digits_per_value() * (3 + h->n_constr)));
+    CKC(h, cudaMemset(h->rzd, 0, sizeof(long long) * 5 * h->n_loc_cols));
+    CKC(h, cudaMemset(h->rsd, 0, sizeof(long long) * (15 + 5 * h->n_constr)));
+  }
+  h->repro = on != 0;
+  h->initialized = false;
   return LSQR_OK;
 }
 
@@ -904,6 +938,18 @@ int lsqr_init(lsqr_t h, const lsqr_solve_params* p) {
   CKC(h, cudaMemcpyAsync(h->st, &st0, sizeof st0, cudaMemcpyHostToDevice, h->s));
   for (double* q : {h->v, h->w, h->x, h->var}) CKL(h, launch_fill(q, h->n_loc_cols, 0.0, h->s), "fill");
   CKL(h, launch_fill(h->zsh, h->n_sh + 8, 0.0, h->s), "fill");
+  if (h->repro) {  // NEXT-4 O-1
+    CKC(h, cudaMemsetAsync(h->rzd, 0, sizeof(long long) * 5 * h->n_loc_cols, h->s));
+    CKC(h, cudaMemsetAsync(h->rsd, 0, sizeof(long long) * (15 + 5 * h->n_constr), h->s));
+    CKL(h, repro_iteration(S, h->u, h->uc, h->crhs, h->v, h->w, h->x, h->var, h->rzd, h->rsd, h->st, h->hflag_dev,
+                           1, h->s), "repro_init");
+    h->b_valid = false;
+    h->initialized = true;
+    if (p->use_graph) CKR(build_graph(h));
+    else if (h->gexec) { cudaGraphExecDestroy(h->gexec); h->gexec = nullptr; h->graph_ok = false; }
+    leave(h);
+    return LSQR_OK;
+  }
   // O-1: u = b, beta = ||u|| (constraint rows: u_c = rhs)
   CKL(h, launch_sumsq(h->u, h->n_loc_rows, h->part_g1, kG1, h->s), "sumsq");
   if (!multi) {
@@ -1026,7 +1072,12 @@ int lsqr_get_state(lsqr_t h, double* sc, double* u, double* v, double* w, double
   if (u) {
     CKC(h, cudaMemcpy(u, h->u, sizeof(double) * h->n_loc_rows, cudaMemcpyDeviceToHost));
     for (int64_t i = 0; i < h->n_loc_rows; ++i) u[i] *= st.inv_beta;
-    if (h->n_constr) CKC(h, cudaMemcpy(u + h->n_loc_rows, h->ucn, sizeof(double) * h->n_constr, cudaMemcpyDeviceToHost));
+    if (h->n_constr) {
+      CKC(h, cudaMemcpy(u + h->n_loc_rows, h->repro ? h->uc : h->ucn, sizeof(double) * h->n_constr,
+                        cudaMemcpyDeviceToHost));
+      if (h->repro)  // repro mode keeps the constraint u unnormalised too
+        for (int64_t k = 0; k < h->n_constr; ++k) u[h->n_loc_rows + k] *= st.inv_beta;
+    }
   }
   const size_t nb = sizeof(double) * h->n_loc_cols;
   if (v) CKC(h, cudaMemcpy(v, h->v, nb, cudaMemcpyDeviceToHost));

@@ -82,6 +82,7 @@ struct DevState {
   double t1, t2, t3; // x += t1 w ; w = v + t2 w ; d = t3 w
   double rn_tmp;
   double pb_beta, pb_ib;  // k_post -> k_scalar hand-over (written by k_post block 0, read by k_scalar only)
+  double r_rho, r_theta, r_phi, r_sn;  // repro mode: k_r_scalar_a -> k_r_scalar_b hand-over
   int32_t itn, istop, istop_first, itn_limit;
   int32_t fixed_count, halted, col_enable, v_pending, beta_pos, pb_pos, pad_[2];
 };
@@ -169,5 +170,15 @@ cudaError_t launch_precond_D(double* c, int64_t n, cudaStream_t s);
 cudaError_t launch_finalize(const double* x, const double* var, const double* D, int64_t n, const DevState* st,
                             double se_t, double* x_out, double* se_out, cudaStream_t s);
 cudaError_t launch_fill(double* p, int64_t n, double v, cudaStream_t s);
+
+// NEXT-4 bitwise-reproducible mode (lsqr_repro.cu, docs/REPRO.md).  Digit buffers: zd [n_cols][5] (zeroed; left
+// zeroed), sd [15 + 5 n_constr] (beta^2 | alpha^2 | ddnorm | constraint rows; zeroed, left zeroed).  u / uc hold
+// u_hat (unnormalised) like the default path; st->inv_beta normalises.
+int64_t repro_digits_per_value();
+cudaError_t repro_iteration(const SysView& S, double* u, double* uc, const double* crhs, double* v, double* w,
+                            double* x, double* var, long long* zd, long long* sd, DevState* st, int32_t* host_flag,
+                            int init, cudaStream_t s);
+// D_j = 1/sqrt(round(EDA sum a_ij^2)) (1 if 0) over the local rows and owned constraint entries (single rank)
+cudaError_t repro_colnorm_D(const SysView& S, double* D, long long* zd, cudaStream_t s);
 
 }  // namespace lsqr

@@ -1,0 +1,440 @@
+// lsqr_repro.cu -- bitwise-reproducible mode (docs/REPRO.md), product side.
+//
+// Every reduction is an exact digit accumulation (EDA: 5 signed 40-bit digits over bits [-168, 32)) of identically
+// rounded FP64 terms, combined with 64-bit integer additions/atomics, which are associative: the result does not
+// depend on thread, warp, block or atomic order.  Every other operation is a single IEEE operation written with
+// explicit _rn intrinsics (no FMA contraction), in the order the Paige-Saunders recurrence writes them.  The CPU
+// oracle implements the same spec independently (oracle/avugsr_oracle.c), so iterates agree bit for bit.
+//
+// These kernels are simple (thread per row / column, global atomics for every digit): the mode is for verification
+// and run-to-run reproducibility, not for speed.
+#include "lsqr_internal.cuh"
+
+namespace lsqr {
+
+namespace {
+
+constexpr int kL = 5;  // digits
+__device__ __constant__ int kB[kL] = {-8, -48, -88, -128, -168};
+
+struct Eda {
+  long long d[kL];
+};
+
+__device__ __forceinline__ void eda_zero(Eda& A) {
+#pragma unroll
+  for (int q = 0; q < kL; ++q) A.d[q] = 0;
+}
+
+// split c into digits and add them (docs/REPRO.md "split")
+__device__ __forceinline__ void eda_add(Eda& A, double c) {
+  const unsigned long long bits = (unsigned long long)__double_as_longlong(c);
+  const bool neg = (bits >> 63) != 0;
+  const int ex = (int)((bits >> 52) & 0x7ff);
+  unsigned long long M = bits & ((1ull << 52) - 1);
+  int E;
+  if (ex == 0) {
+    E = -1074;
+  } else {
+    M |= 1ull << 52;
+    E = ex - 1075;
+  }
+  if (M == 0) return;
+#pragma unroll
+  for (int q = 0; q < kL; ++q) {
+    const int sh = E - kB[q];
+    unsigned long long dig;
+    if (sh >= 40) dig = 0;
+    else if (sh >= 0) dig = (M << sh) & ((1ull << 40) - 1);
+    else if (sh > -53) dig = (M >> (-sh)) & ((1ull << 40) - 1);
+    else dig = 0;
+    A.d[q] += neg ? -(long long)dig : (long long)dig;
+  }
+}
+
+__device__ __forceinline__ double eda_round_d(const long long* Din) {
+  long long D[kL];
+#pragma unroll
+  for (int q = 0; q < kL; ++q) D[q] = Din[q];
+#pragma unroll
+  for (int q = kL - 1; q >= 1; --q) {
+    const long long c = D[q] >> 40;  // arithmetic shift = floor division
+    D[q] -= c * (1ll << 40);
+    D[q - 1] += c;
+  }
+  const double pw[kL] = {0x1p-8, 0x1p-48, 0x1p-88, 0x1p-128, 0x1p-168};
+  double v = 0.0;
+#pragma unroll
+  for (int q = 0; q < kL; ++q) v = __dadd_rn(v, __dmul_rn(__ll2double_rn(D[q]), pw[q]));
+  return v;
+}
+
+// integer reduction of a thread's digits over the block, then one 64-bit atomic per digit (exact, order-free)
+__device__ __forceinline__ void eda_flush_block(const Eda& A, long long* __restrict__ dst) {
+  __shared__ long long sd[kL][kRedThreads / 32];
+#pragma unroll
+  for (int q = 0; q < kL; ++q) {
+    long long v = A.d[q];
+#pragma unroll
+    for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if ((threadIdx.x & 31) == 0) sd[q][threadIdx.x >> 5] = v;
+  }
+  __syncthreads();
+  if (threadIdx.x < kL) {
+    long long t = 0;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += sd[threadIdx.x][w];
+    if (t != 0) atomicAdd(reinterpret_cast<unsigned long long*>(dst + threadIdx.x), (unsigned long long)t);
+  }
+  __syncthreads();
+}
+
+__device__ __forceinline__ void eda_atomic(long long* __restrict__ dst, const Eda& A) {
+#pragma unroll
+  for (int q = 0; q < kL; ++q)
+    if (A.d[q] != 0) atomicAdd(reinterpret_cast<unsigned long long*>(dst + q), (unsigned long long)A.d[q]);
+}
+
+__device__ __forceinline__ void ic_cols(const SysView& S, const IdxRec& r, int64_t star, int64_t (&col)[kSlots]) {
+  // column of every slot (paper order): astro 0-4, attitude 5-16, instrumental 17-22, global 23
+  for (int a = 0; a < 5; ++a) col[a] = 5 * star + a;
+  for (int t = 0; t < 12; ++t) col[5 + t] = S.A0 + (int64_t)(t / 4) * S.n_axis + r.k0 + (t % 4);
+  const uint32_t w3[3] = {r.ic01, r.ic23, r.ic45};
+  for (int q = 0; q < 6; ++q) col[17 + q] = S.I0 + S.ip.inv((w3[q / 2] >> ((q & 1) * 16)) & 0xffffu);
+  col[23] = S.G0;
+}
+
+__device__ __forceinline__ int64_t star_of(const SysView& S, int64_t row) {
+  int64_t lo = 0, hi = S.n_stars;  // star_ptr[lo] <= row < star_ptr[hi]
+  while (hi - lo > 1) {
+    const int64_t mid = (lo + hi) >> 1;
+    if (S.star_ptr[mid] <= row) lo = mid;
+    else hi = mid;
+  }
+  return lo;
+}
+
+// value of paper slot sl of local row `row` (rows are stored lane-major: position 6j+t holds slot_of(t, j))
+__device__ __forceinline__ void row_vals(const SysView& S, int64_t row, double (&v)[kSlots]) {
+  const double* rp = S.vals + row * kSlots;
+  for (int p = 0; p < kSlots; ++p) v[slot_of(p % 6, p / 6)] = rp[p];
+}
+
+// ---------------------------------------------------------------------------------------------------- kernels
+// aprod1 (P&S step a): u_hat_i <- ((-alpha) * (ib * u_hat_i)) + round(EDA_s a_is * v[col_is]); beta^2 digits.
+__global__ void k_r_aprod1(SysView S, const double* __restrict__ v, double* __restrict__ u, long long* __restrict__ b2d,
+                           long long* __restrict__ cd, const DevState* __restrict__ st, int init) {
+  if (!init && st->halted) return;
+  const double ib = st->inv_beta, nalpha = -st->alpha;
+  Eda B;
+  eda_zero(B);
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < S.n_rows; i += (int64_t)gridDim.x * blockDim.x) {
+    if (init) {  // u = b: beta^2 of b
+      eda_add(B, __dmul_rn(u[i], u[i]));
+      continue;
+    }
+    double val[kSlots];
+    int64_t col[kSlots];
+    row_vals(S, i, val);
+    ic_cols(S, S.idx[i], star_of(S, i), col);
+    Eda A;
+    eda_zero(A);
+    for (int sl = 0; sl < kSlots; ++sl) {
+      if (sl == 23 && S.n_glob == 0) continue;
+      eda_add(A, __dmul_rn(val[sl], v[col[sl]]));
+    }
+    const double un = __dadd_rn(__dmul_rn(nalpha, __dmul_rn(ib, u[i])), eda_round_d(A.d));
+    u[i] = un;
+    eda_add(B, __dmul_rn(un, un));
+  }
+  eda_flush_block(B, b2d);
+  if (init) return;
+  // constraint rows: digits of every owned entry's product, one thread per chunk (chunks lie within one row)
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < S.n_chunks; q += (int64_t)gridDim.x * blockDim.x) {
+    Eda A;
+    eda_zero(A);
+    for (int64_t e = S.ch_beg[q]; e < S.ch_end[q]; ++e) eda_add(A, __dmul_rn(S.cval[e], v[S.ccol[e]]));
+    eda_atomic(cd + (int64_t)S.ch_row[q] * kL, A);
+  }
+}
+
+// beta (one thread): constraint u, ||u||, anorm (P&S step b bookkeeping); resets the digit accumulators it read
+__global__ void k_r_beta(SysView S, long long* __restrict__ b2d, long long* __restrict__ cd, double* __restrict__ uc,
+                         const double* __restrict__ crhs, DevState* __restrict__ st, int init) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  if (!init && st->halted) return;
+  Eda B;
+  for (int q = 0; q < kL; ++q) B.d[q] = b2d[q];
+  const double ib = st->inv_beta, nalpha = -st->alpha;
+  for (int k = 0; k < S.n_constr; ++k) {
+    double un;
+    if (init) {
+      un = crhs ? crhs[k] : 0.0;
+    } else {
+      un = __dadd_rn(__dmul_rn(nalpha, __dmul_rn(ib, uc[k])), eda_round_d(cd + (int64_t)k * kL));
+      for (int q = 0; q < kL; ++q) cd[(int64_t)k * kL + q] = 0;
+    }
+    uc[k] = un;
+    eda_add(B, __dmul_rn(un, un));
+  }
+  for (int q = 0; q < kL; ++q) b2d[q] = 0;
+  const double beta = __dsqrt_rn(eda_round_d(B.d));
+  const int pos = beta > 0.0;
+  if (init) {
+    st->bnorm = beta;
+  } else if (pos) {
+    const double a = st->alpha, d = st->damp;
+    st->anorm = __dsqrt_rn(
+        __dadd_rn(__dadd_rn(__dadd_rn(__dmul_rn(st->anorm, st->anorm), __dmul_rn(a, a)), __dmul_rn(beta, beta)),
+                  __dmul_rn(d, d)));
+  }
+  st->beta = beta;
+  st->beta_pos = pos;
+  st->inv_beta = pos ? __ddiv_rn(1.0, beta) : 1.0;
+}
+
+// aprod2 contributions: digits of a_ij * (ib * u_hat_i) into zd[col] (all columns), constraint entries likewise
+__global__ void k_r_aprod2(SysView S, const double* __restrict__ u, const double* __restrict__ uc,
+                           long long* __restrict__ zd, const DevState* __restrict__ st, int colnorm) {
+  if (!colnorm && (st->halted || !st->beta_pos)) return;
+  const double ib = colnorm ? 1.0 : st->inv_beta;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < S.n_rows; i += (int64_t)gridDim.x * blockDim.x) {
+    double val[kSlots];
+    int64_t col[kSlots];
+    row_vals(S, i, val);
+    ic_cols(S, S.idx[i], star_of(S, i), col);
+    const double y = colnorm ? 0.0 : __dmul_rn(ib, u[i]);
+    for (int sl = 0; sl < kSlots; ++sl) {
+      if (sl == 23 && S.n_glob == 0) continue;
+      Eda A;
+      eda_zero(A);
+      eda_add(A, colnorm ? __dmul_rn(val[sl], val[sl]) : __dmul_rn(val[sl], y));
+      eda_atomic(zd + col[sl] * kL, A);
+    }
+  }
+  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < S.n_chunks; q += (int64_t)gridDim.x * blockDim.x) {
+    const double yc = colnorm ? 0.0 : __dmul_rn(ib, uc[S.ch_row[q]]);
+    for (int64_t e = S.ch_beg[q]; e < S.ch_end[q]; ++e) {
+      const double cv = S.cval[e];
+      Eda A;
+      eda_zero(A);
+      eda_add(A, colnorm ? __dmul_rn(cv, cv) : __dmul_rn(cv, yc));
+      eda_atomic(zd + S.ccol[e] * kL, A);
+    }
+  }
+}
+
+// v_j <- ((-beta) * v_j) + round(zd_j) on every column (init: v_j = 0 + round(zd_j)); alpha^2 digits; zd reset.
+// colnorm: D_j = 1/sqrt(c_j) (1 if c_j == 0) with c_j = round(zd_j).
+__global__ void k_r_vupdate(int64_t n, double* __restrict__ v, long long* __restrict__ zd, long long* __restrict__ a2d,
+                            const DevState* __restrict__ st, int mode) {  // mode 0 LSQR, 1 init, 2 colnorm -> D
+  if (mode == 0 && (st->halted || !st->beta_pos)) return;
+  if (mode == 1 && !st->beta_pos) return;
+  const double nbeta = mode == 2 ? 0.0 : -st->beta;
+  Eda A;
+  eda_zero(A);
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x) {
+    const double z = eda_round_d(zd + c * kL);
+#pragma unroll
+    for (int q = 0; q < kL; ++q) zd[c * kL + q] = 0;
+    if (mode == 2) {
+      v[c] = z > 0.0 ? __ddiv_rn(1.0, __dsqrt_rn(z)) : 1.0;
+      continue;
+    }
+    const double vn = mode == 1 ? __dadd_rn(v[c], z) : __dadd_rn(__dmul_rn(nbeta, v[c]), z);
+    v[c] = vn;
+    eda_add(A, __dmul_rn(vn, vn));
+  }
+  if (mode != 2) eda_flush_block(A, a2d);
+}
+
+// P&S steps b (alpha), c, d (rotation): t1, t2, t3 -- one thread
+__global__ void k_r_scalar_a(DevState* __restrict__ st, long long* __restrict__ a2d, int init, int32_t* __restrict__ host_flag) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  if (!init && st->halted) {
+    st->col_enable = 0;
+    return;
+  }
+  const int bp = st->beta_pos;
+  double alpha = st->alpha;
+  if (bp) {
+    alpha = __dsqrt_rn(eda_round_d(a2d));
+    st->inv_alpha = alpha > 0.0 ? __ddiv_rn(1.0, alpha) : 1.0;
+    st->v_pending = 1;
+  } else {
+    st->v_pending = 0;
+  }
+  for (int q = 0; q < kL; ++q) a2d[q] = 0;
+  st->alpha = alpha;
+  st->col_enable = 1;
+  if (init) {  // O-1/O-2
+    const double beta = st->beta;
+    st->rhobar = alpha; st->phibar = beta; st->rnorm = beta; st->r1norm = beta; st->r2norm = beta;
+    st->anorm = 0; st->acond = 0; st->ddnorm = 0; st->res2 = 0; st->xnorm = 0; st->xxnorm = 0; st->z = 0;
+    st->cs2 = -1.0; st->sn2 = 0.0;
+    st->arnorm = __dmul_rn(alpha, beta);
+    st->t1 = 0.0; st->t2 = 0.0; st->t3 = 0.0;
+    st->itn = 0; st->istop = 0; st->istop_first = 0;
+    st->halted = (st->arnorm == 0.0) ? 1 : 0;
+    if (host_flag) *reinterpret_cast<volatile int32_t*>(host_flag) = st->halted;
+    return;
+  }
+  st->itn += 1;
+  const double beta = st->beta, damp = st->damp, dampsq = __dmul_rn(damp, damp);
+  double rhobar = st->rhobar, phibar = st->phibar, psi, rhobar1;
+  if (damp > 0.0) {
+    rhobar1 = __dsqrt_rn(__dadd_rn(__dmul_rn(rhobar, rhobar), dampsq));
+    const double cs1 = __ddiv_rn(rhobar, rhobar1), sn1 = __ddiv_rn(damp, rhobar1);
+    psi = __dmul_rn(sn1, phibar);
+    phibar = __dmul_rn(cs1, phibar);
+  } else {
+    rhobar1 = rhobar;
+    psi = 0.0;
+  }
+  const double rho = __dsqrt_rn(__dadd_rn(__dmul_rn(rhobar1, rhobar1), __dmul_rn(beta, beta)));
+  const double cs = __ddiv_rn(rhobar1, rho), sn = __ddiv_rn(beta, rho);
+  const double theta = __dmul_rn(sn, alpha);
+  st->rhobar = __dmul_rn(-cs, alpha);
+  const double phi = __dmul_rn(cs, phibar);
+  st->phibar = __dmul_rn(sn, phibar);
+  st->rn_tmp = psi;  // carried to scalar_b
+  st->t1 = __ddiv_rn(phi, rho);
+  st->t2 = __ddiv_rn(-theta, rho);
+  st->t3 = __ddiv_rn(1.0, rho);
+  st->r_rho = rho;  // hand-over to scalar_b
+  st->r_theta = theta;
+  st->r_phi = phi;
+  st->r_sn = sn;
+}
+
+// O-3e: v <- (1/alpha) v (if pending); d = t3 w; var += d*d; x += t1 w; w = v + t2 w; ddnorm digits
+__global__ void k_r_colupdate(double* __restrict__ v, double* __restrict__ w, double* __restrict__ x,
+                              double* __restrict__ var, int64_t n, long long* __restrict__ ddd,
+                              const DevState* __restrict__ st, int init) {
+  if (!st->col_enable) return;
+  const double ia = st->inv_alpha, t1 = st->t1, t2 = st->t2, t3 = st->t3;
+  const int vp = st->v_pending && st->alpha > 0.0;
+  Eda A;
+  eda_zero(A);
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const double vi = vp ? __dmul_rn(ia, v[i]) : v[i];
+    v[i] = vi;
+    if (init) {  // w = v
+      w[i] = vi;
+      continue;
+    }
+    const double wi = w[i];
+    const double dk = __dmul_rn(t3, wi);
+    const double d2 = __dmul_rn(dk, dk);
+    var[i] = __dadd_rn(var[i], d2);
+    eda_add(A, d2);
+    x[i] = __dadd_rn(x[i], __dmul_rn(t1, wi));
+    w[i] = __dadd_rn(vi, __dmul_rn(t2, wi));
+  }
+  if (!init) eda_flush_block(A, ddd);
+}
+
+// O-3f-j after the column update (ddnorm needed by acond) -- one thread
+__global__ void k_r_scalar_b(DevState* __restrict__ st, long long* __restrict__ ddd, int32_t* __restrict__ host_flag) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  if (st->halted || !st->col_enable) return;
+  const double eps = 0x1p-52;
+  const double rho = st->r_rho, theta = st->r_theta, phi = st->r_phi, sn = st->r_sn, psi = st->rn_tmp;
+  const double tau = __dmul_rn(sn, phi);
+  const double ddnorm = __dadd_rn(st->ddnorm, eda_round_d(ddd));
+  for (int q = 0; q < kL; ++q) ddd[q] = 0;
+  // f.
+  const double delta = __dmul_rn(st->sn2, rho), gambar = __dmul_rn(-st->cs2, rho);
+  const double rhs = __dadd_rn(phi, -__dmul_rn(delta, st->z));
+  const double zbar = __ddiv_rn(rhs, gambar);
+  const double xnorm = __dsqrt_rn(__dadd_rn(st->xxnorm, __dmul_rn(zbar, zbar)));
+  const double gamma = __dsqrt_rn(__dadd_rn(__dmul_rn(gambar, gambar), __dmul_rn(theta, theta)));
+  st->cs2 = __ddiv_rn(gambar, gamma);
+  st->sn2 = __ddiv_rn(theta, gamma);
+  st->z = __ddiv_rn(rhs, gamma);
+  st->xxnorm = __dadd_rn(st->xxnorm, __dmul_rn(st->z, st->z));
+  // g.
+  const double anorm = st->anorm, damp = st->damp, dampsq = __dmul_rn(damp, damp);
+  const double acond = __dmul_rn(anorm, __dsqrt_rn(ddnorm));
+  const double res2 = __dadd_rn(st->res2, __dmul_rn(psi, psi));
+  const double phibar = st->phibar;
+  const double rnorm = __dsqrt_rn(__dadd_rn(__dmul_rn(phibar, phibar), res2));
+  const double arnorm = __dmul_rn(st->alpha, fabs(tau));
+  double r1norm;
+  if (damp > 0.0) {
+    const double r1sq = __dadd_rn(__dmul_rn(rnorm, rnorm), -__dmul_rn(dampsq, st->xxnorm));
+    r1norm = __dsqrt_rn(fabs(r1sq));
+    if (r1sq < 0) r1norm = -r1norm;
+  } else {
+    r1norm = rnorm;
+  }
+  // h.
+  const double bnorm = st->bnorm;
+  const double test1 = __ddiv_rn(rnorm, bnorm);
+  const double test2 = __ddiv_rn(arnorm, __dadd_rn(__dmul_rn(anorm, rnorm), eps));
+  const double test3 = __ddiv_rn(1.0, __dadd_rn(acond, eps));
+  const double axb = __ddiv_rn(__dmul_rn(anorm, xnorm), bnorm);
+  const double tt1 = __ddiv_rn(test1, __dadd_rn(1.0, axb));
+  const double rtol = __dadd_rn(st->btol, __ddiv_rn(__dmul_rn(__dmul_rn(st->atol, anorm), xnorm), bnorm));
+  // i.
+  int is = 0;
+  if (st->itn >= st->itn_limit) is = 7;
+  if (__dadd_rn(1.0, test3) <= 1.0) is = 6;
+  if (__dadd_rn(1.0, test2) <= 1.0) is = 5;
+  if (__dadd_rn(1.0, tt1) <= 1.0) is = 4;
+  if (test3 <= st->ctol) is = 3;
+  if (test2 <= st->atol) is = 2;
+  if (test1 <= rtol) is = 1;
+  st->ddnorm = ddnorm; st->xnorm = xnorm; st->acond = acond; st->res2 = res2; st->rnorm = rnorm;
+  st->r1norm = r1norm; st->r2norm = rnorm; st->arnorm = arnorm;
+  st->istop = is;
+  if (is != 0 && st->istop_first == 0) st->istop_first = is;
+  if ((is != 0 && !st->fixed_count) || st->itn >= st->itn_limit) st->halted = 1;
+  if (host_flag) *reinterpret_cast<volatile int32_t*>(host_flag) = st->halted | (st->itn << 1);
+}
+
+int grid_for(int64_t n) {
+  int64_t b = (n + kRedThreads - 1) / kRedThreads;
+  if (b < 1) b = 1;
+  return (int)(b < 148 * 8 ? b : 148 * 8);
+}
+
+}  // namespace
+
+int64_t repro_digits_per_value() { return kL; }
+
+cudaError_t repro_iteration(const SysView& S, double* u, double* uc, const double* crhs, double* v, double* w,
+                            double* x, double* var, long long* zd, long long* sd, DevState* st, int32_t* host_flag,
+                            int init, cudaStream_t s) {
+  long long* b2d = sd;       // beta^2 digits
+  long long* a2d = sd + kL;  // alpha^2 digits
+  long long* ddd = sd + 2 * kL;
+  long long* cd = sd + 3 * kL;  // constraint row digits [n_constr][kL]
+  const int gr = grid_for(S.n_rows > S.n_chunks ? S.n_rows : S.n_chunks);
+  const int gc = grid_for(S.n_cols);
+  if (init) {
+    k_r_aprod1<<<gr, kRedThreads, 0, s>>>(S, v, u, b2d, cd, st, 1);
+    k_r_beta<<<1, 32, 0, s>>>(S, b2d, cd, uc, crhs, st, 1);
+    k_r_aprod2<<<gr, kRedThreads, 0, s>>>(S, u, uc, zd, st, 0);
+    k_r_vupdate<<<gc, kRedThreads, 0, s>>>(S.n_cols, v, zd, a2d, st, 1);
+    k_r_scalar_a<<<1, 32, 0, s>>>(st, a2d, 1, host_flag);
+    k_r_colupdate<<<gc, kRedThreads, 0, s>>>(v, w, x, var, S.n_cols, ddd, st, 1);
+    return cudaGetLastError();
+  }
+  k_r_aprod1<<<gr, kRedThreads, 0, s>>>(S, v, u, b2d, cd, st, 0);
+  k_r_beta<<<1, 32, 0, s>>>(S, b2d, cd, uc, crhs, st, 0);
+  k_r_aprod2<<<gr, kRedThreads, 0, s>>>(S, u, uc, zd, st, 0);
+  k_r_vupdate<<<gc, kRedThreads, 0, s>>>(S.n_cols, v, zd, a2d, st, 0);
+  k_r_scalar_a<<<1, 32, 0, s>>>(st, a2d, 0, nullptr);
+  k_r_colupdate<<<gc, kRedThreads, 0, s>>>(v, w, x, var, S.n_cols, ddd, st, 0);
+  k_r_scalar_b<<<1, 32, 0, s>>>(st, ddd, host_flag);
+  return cudaGetLastError();
+}
+
+cudaError_t repro_colnorm_D(const SysView& S, double* D, long long* zd, cudaStream_t s) {
+  const int gr = grid_for(S.n_rows > S.n_chunks ? S.n_rows : S.n_chunks);
+  k_r_aprod2<<<gr, kRedThreads, 0, s>>>(S, nullptr, nullptr, zd, nullptr, 1);
+  k_r_vupdate<<<grid_for(S.n_cols), kRedThreads, 0, s>>>(S.n_cols, D, zd, nullptr, nullptr, 2);
+  return cudaGetLastError();
+}
+
+}  // namespace lsqr

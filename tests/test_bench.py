@@ -52,3 +52,10 @@ def test_bench_two_ranks_gloo_callback(cuda_device):
     assert d["config"]["n_obs_per_gpu"] == 20_000 and d["config"]["total_rows"] == 40_000
     assert d["config"]["parallelism"].startswith("dp2")
     assert d["gpu_launches"] == 4 * 9
+
+
+@pytest.mark.gpu
+def test_bench_repro_line(cuda_device):
+    d = _run(["bench.py", "--config", "C1", "--steps", "4", "--warmup", "3", "--repro", "--cpu-iters", "1"])
+    assert d["gpu_launches"] == 4 * 7 and "reproducible" in d["config"]["variant"]
+    assert d["roofline"]["kernel"] == "repro iteration" and "repro" in d["cpu_baseline"]["sample"]

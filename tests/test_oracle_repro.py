@@ -107,3 +107,17 @@ def test_repro_products_vs_dense():
     yy = rng.standard_normal(S.m_local)
     xx = np.zeros(S.n_cols); S.aprod2_repro(yy, xx)
     assert np.allclose(xx, A.T @ yy, rtol=1e-15, atol=1e-15)
+
+
+def test_repro_colnorms_exact_and_permutation_invariant():
+    """NEXT-4 preconditioner: c_j = round(EDA sum a_ij^2) equals the exact rational sum of the rounded squares to
+    within 1 ulp, agrees with the ordered fp64 sum, and is bitwise invariant under row permutation."""
+    S = oracle.System(W.micro(n_stars=11, obs=25, n_ext=4, seed=13))
+    c = S.colnorms(repro=True)
+    A = S.dense()
+    for j in range(S.n_cols):
+        ex = sum((Fraction(float(a * a)) for a in A[:, j]), Fraction(0))
+        assert abs(Fraction(c[j]) - ex) <= Fraction(abs(c[j])) * Fraction(2) ** -52
+    assert np.allclose(c, S.colnorms(), rtol=1e-14, atol=0)
+    P, _ = permuted(S, np.random.default_rng(8))
+    assert np.array_equal(P.colnorms(repro=True), c)

@@ -1,5 +1,5 @@
 """Small end-to-end run used under compute-sanitizer (tests/test_sanitizer.py): generate, precondition, products,
-two solves (fused and two-pass), set_system round trip.  Exits non-zero on any library error."""
+two solves (fused and two-pass), set_system round trip, and the bitwise-reproducible mode (NEXT-4).  Exits non-zero on any library error."""
 import os
 import sys
 
@@ -28,6 +28,12 @@ def main():
         s.set_system(g["vals"], g["mA"], g["mT"], g["iC"], g["b"])
         out = s.solve(itn_limit=3, fused=fused, use_graph=True)
         s.close()
+    s = avu.Solver.synthetic(w, torch_alloc=False)
+    s.set_reproducible(True)
+    s.precondition()
+    out = s.solve(itn_limit=6, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=False)
+    assert out["itn"] == 6 and np.isfinite(out["x"]).all()
+    s.close()
     torch.cuda.synchronize()
     print("sanitize run ok")
 
