@@ -249,7 +249,7 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   const bool fused = h->params.fused != 0;
   if (h->repro) {  // NEXT-4: 7 launches, all in lsqr_repro.cu
     if (ev) cudaEventRecord(ev[0], s);
-    CKL(h, repro_iteration(S, h->u, h->uc, h->crhs, h->v, h->w, h->x, h->var, h->rzd, h->rsd, h->st, h->hflag_dev,
+    CKL(h, repro_iteration(S, h->grid, h->u, h->uc, h->crhs, h->v, h->w, h->x, h->var, h->rzd, h->rsd, h->st, h->hflag_dev,
                            0, s), "repro");
     if (ev) for (int k = 1; k < 4; ++k) cudaEventRecord(ev[k], s);
     return LSQR_OK;
@@ -838,7 +838,7 @@ int lsqr_precondition(lsqr_t h) {
   SysView& S = h->S;
   enter(h);
   if (h->repro) {  // NEXT-4: exact column sums of squares
-    CKL(h, repro_colnorm_D(S, h->D, h->rzd, h->s), "colnorm_repro");
+    CKL(h, repro_colnorm_D(S, h->grid, h->D, h->rzd, h->s), "colnorm_repro");
     CKL(h, launch_scale_rows(S, h->grid, h->vals, h->D, h->s), "scale_rows");
     CKL(h, launch_scale_constr(S, const_cast<double*>(S.cval), h->D, h->s), "scale_constr");
     leave(h);
@@ -941,7 +941,7 @@ int lsqr_init(lsqr_t h, const lsqr_solve_params* p) {
   if (h->repro) {  // NEXT-4 O-1
     CKC(h, cudaMemsetAsync(h->rzd, 0, sizeof(long long) * 5 * h->n_loc_cols, h->s));
     CKC(h, cudaMemsetAsync(h->rsd, 0, sizeof(long long) * (15 + 5 * h->n_constr), h->s));
-    CKL(h, repro_iteration(S, h->u, h->uc, h->crhs, h->v, h->w, h->x, h->var, h->rzd, h->rsd, h->st, h->hflag_dev,
+    CKL(h, repro_iteration(S, h->grid, h->u, h->uc, h->crhs, h->v, h->w, h->x, h->var, h->rzd, h->rsd, h->st, h->hflag_dev,
                            1, h->s), "repro_init");
     h->b_valid = false;
     h->initialized = true;

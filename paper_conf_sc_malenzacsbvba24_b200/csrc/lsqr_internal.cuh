@@ -171,14 +171,15 @@ cudaError_t launch_finalize(const double* x, const double* var, const double* D,
                             double se_t, double* x_out, double* se_out, cudaStream_t s);
 cudaError_t launch_fill(double* p, int64_t n, double v, cudaStream_t s);
 
-// NEXT-4 bitwise-reproducible mode (lsqr_repro.cu, docs/REPRO.md).  Digit buffers: zd [n_cols][5] (zeroed; left
-// zeroed), sd [15 + 5 n_constr] (beta^2 | alpha^2 | ddnorm | constraint rows; zeroed, left zeroed).  u / uc hold
-// u_hat (unnormalised) like the default path; st->inv_beta normalises.
+// NEXT-4 bitwise-reproducible mode (lsqr_repro.cu, docs/REPRO.md).  Digit buffers: zd [5][n_cols] (digit-major; zeroed;
+// left zeroed), sd [15 + 5 n_constr] (beta^2 | alpha^2 | ddnorm | constraint rows; zeroed, left zeroed).  u / uc hold
+// u_hat (unnormalised) like the default path; st->inv_beta normalises.  grid: the persistent row-kernel grid
+// (kThreads per CTA) that SysView::warp_star partitions.
 int64_t repro_digits_per_value();
-cudaError_t repro_iteration(const SysView& S, double* u, double* uc, const double* crhs, double* v, double* w,
+cudaError_t repro_iteration(const SysView& S, int grid, double* u, double* uc, const double* crhs, double* v, double* w,
                             double* x, double* var, long long* zd, long long* sd, DevState* st, int32_t* host_flag,
                             int init, cudaStream_t s);
 // D_j = 1/sqrt(round(EDA sum a_ij^2)) (1 if 0) over the local rows and owned constraint entries (single rank)
-cudaError_t repro_colnorm_D(const SysView& S, double* D, long long* zd, cudaStream_t s);
+cudaError_t repro_colnorm_D(const SysView& S, int grid, double* D, long long* zd, cudaStream_t s);
 
 }  // namespace lsqr

@@ -26,29 +26,57 @@ __device__ __forceinline__ void eda_zero(Eda& A) {
   for (int q = 0; q < kL; ++q) A.d[q] = 0;
 }
 
-// split c into digits and add them (docs/REPRO.md "split")
-__device__ __forceinline__ void eda_add(Eda& A, double c) {
-  const unsigned long long bits = (unsigned long long)__double_as_longlong(c);
-  const bool neg = (bits >> 63) != 0;
+// split(c) (docs/REPRO.md): with p = E - B_4 the offset of the significand's lowest bit above the window bottom, the
+// significand lands in digits 4-k, 3-k, 2-k (k = p div 40) as the 40-bit pieces lo, mid, hi of M << (p mod 40); bits
+// below the window (p < 0) are truncated first, pieces above digit 0 are dropped.  These are exactly the digits of
+// the spec's per-digit rule (at most three of them nonzero).
+struct Pieces {
+  long long lo, mid, hi;
+  int k;
+};
+
+__device__ __forceinline__ Pieces eda_split(double c) {
+  const long long bits = __double_as_longlong(c);
   const int ex = (int)((bits >> 52) & 0x7ff);
-  unsigned long long M = bits & ((1ull << 52) - 1);
-  int E;
-  if (ex == 0) {
-    E = -1074;
-  } else {
-    M |= 1ull << 52;
-    E = ex - 1075;
+  unsigned long long M = (unsigned long long)bits & ((1ull << 52) - 1);
+  if (ex) M |= 1ull << 52;
+  int p = (ex ? ex - 1075 : -1074) + 168;
+  if (p < 0) {  // (rare) truncate the bits below 2^-168
+    M = p > -53 ? (M >> (-p)) : 0ull;
+    p = 0;
   }
-  if (M == 0) return;
+  const int k = p / 40, o = p - 40 * k;
+  const unsigned long long mask = (1ull << 40) - 1;
+  const long long sgn = bits >> 63;  // 0 or -1
+  Pieces r;
+  r.k = k;
+  r.lo = ((long long)((M << o) & mask) ^ sgn) - sgn;
+  r.mid = ((long long)((M >> (40 - o)) & mask) ^ sgn) - sgn;
+  r.hi = ((long long)(o > 27 ? (M >> (80 - o)) : 0ull) ^ sgn) - sgn;
+  return r;
+}
+
+__device__ __forceinline__ void eda_add(Eda& A, double c) {
+  const Pieces P = eda_split(c);
+  switch (P.k) {  // constant digit indices keep A in registers; k is nearly warp-uniform for real data
+    case 0: A.d[4] += P.lo; A.d[3] += P.mid; A.d[2] += P.hi; break;
+    case 1: A.d[3] += P.lo; A.d[2] += P.mid; A.d[1] += P.hi; break;
+    case 2: A.d[2] += P.lo; A.d[1] += P.mid; A.d[0] += P.hi; break;
+    case 3: A.d[1] += P.lo; A.d[0] += P.mid; break;
+    case 4: A.d[0] += P.lo; break;
+    default: break;
+  }
+}
+
+// the pieces of one term straight into the digit-major column accumulator zd[q][col] (q = 4-k, 3-k, 2-k)
+__device__ __forceinline__ void eda_atomic_term(long long* __restrict__ zd_col, int64_t stride, double c) {
+  const Pieces P = eda_split(c);
+  const long long pc[3] = {P.lo, P.mid, P.hi};
 #pragma unroll
-  for (int q = 0; q < kL; ++q) {
-    const int sh = E - kB[q];
-    unsigned long long dig;
-    if (sh >= 40) dig = 0;
-    else if (sh >= 0) dig = (M << sh) & ((1ull << 40) - 1);
-    else if (sh > -53) dig = (M >> (-sh)) & ((1ull << 40) - 1);
-    else dig = 0;
-    A.d[q] += neg ? -(long long)dig : (long long)dig;
+  for (int r = 0; r < 3; ++r) {
+    const int q = kL - 1 - P.k - r;
+    if (q >= 0 && pc[r] != 0)
+      atomicAdd(reinterpret_cast<unsigned long long*>(zd_col + q * stride), (unsigned long long)pc[r]);
   }
 }
 
@@ -70,8 +98,8 @@ __device__ __forceinline__ double eda_round_d(const long long* Din) {
 }
 
 // integer reduction of a thread's digits over the block, then one 64-bit atomic per digit (exact, order-free)
-__device__ __forceinline__ void eda_flush_block(const Eda& A, long long* __restrict__ dst) {
-  __shared__ long long sd[kL][kRedThreads / 32];
+__device__ __forceinline__ void eda_flush_block(const Eda& A, long long* __restrict__ dst, int64_t stride = 1) {
+  __shared__ long long sd[kL][32];
 #pragma unroll
   for (int q = 0; q < kL; ++q) {
     long long v = A.d[q];
@@ -83,77 +111,210 @@ __device__ __forceinline__ void eda_flush_block(const Eda& A, long long* __restr
   if (threadIdx.x < kL) {
     long long t = 0;
     for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += sd[threadIdx.x][w];
-    if (t != 0) atomicAdd(reinterpret_cast<unsigned long long*>(dst + threadIdx.x), (unsigned long long)t);
+    if (t != 0 && dst)
+      atomicAdd(reinterpret_cast<unsigned long long*>(dst + threadIdx.x * stride), (unsigned long long)t);
   }
   __syncthreads();
 }
 
-__device__ __forceinline__ void eda_atomic(long long* __restrict__ dst, const Eda& A) {
+__device__ __forceinline__ void eda_atomic(long long* __restrict__ dst, const Eda& A, int64_t stride = 1) {
 #pragma unroll
   for (int q = 0; q < kL; ++q)
-    if (A.d[q] != 0) atomicAdd(reinterpret_cast<unsigned long long*>(dst + q), (unsigned long long)A.d[q]);
+    if (A.d[q] != 0) atomicAdd(reinterpret_cast<unsigned long long*>(dst + q * stride), (unsigned long long)A.d[q]);
 }
 
-__device__ __forceinline__ void ic_cols(const SysView& S, const IdxRec& r, int64_t star, int64_t (&col)[kSlots]) {
-  // column of every slot (paper order): astro 0-4, attitude 5-16, instrumental 17-22, global 23
-  for (int a = 0; a < 5; ++a) col[a] = 5 * star + a;
-  for (int t = 0; t < 12; ++t) col[5 + t] = S.A0 + (int64_t)(t / 4) * S.n_axis + r.k0 + (t % 4);
+// Column of position t (0..5) of lane j of a row (lane-major storage: position 6j+t holds paper slot slot_of(t, j)):
+// t=0 astro j; t=1..3 attitude axis t-1, knot j; t=4 instrumental j; t=5: astro 4 (j=0), instrumental 4/5 (j=1/2),
+// global (j=3).  Returns -1 for the global slot when the system has none.
+__device__ __forceinline__ int64_t lane_col(const SysView& S, const IdxRec& r, int64_t star, int t, int j) {
+  if (t == 0) return 5 * star + j;
+  if (t <= 3) return S.A0 + (int64_t)(t - 1) * S.n_axis + r.k0 + j;
   const uint32_t w3[3] = {r.ic01, r.ic23, r.ic45};
-  for (int q = 0; q < 6; ++q) col[17 + q] = S.I0 + S.ip.inv((w3[q / 2] >> ((q & 1) * 16)) & 0xffffu);
-  col[23] = S.G0;
+  if (t == 4) return S.I0 + S.ip.inv((w3[j >> 1] >> ((j & 1) * 16)) & 0xffffu);
+  if (j == 0) return 5 * star + 4;
+  if (j == 3) return S.n_glob ? S.G0 : -1;
+  const int q = 3 + j;  // instrumental 4 or 5
+  return S.I0 + S.ip.inv((w3[q >> 1] >> ((q & 1) * 16)) & 0xffffu);
 }
 
-__device__ __forceinline__ int64_t star_of(const SysView& S, int64_t row) {
-  int64_t lo = 0, hi = S.n_stars;  // star_ptr[lo] <= row < star_ptr[hi]
-  while (hi - lo > 1) {
-    const int64_t mid = (lo + hi) >> 1;
-    if (S.star_ptr[mid] <= row) lo = mid;
-    else hi = mid;
+// Row partition of the repro product kernels: every warp takes an even, 8-aligned slice of the rows (star ownership
+// is irrelevant here: integer digit sums are exact and associative, so how the terms are grouped -- registers,
+// shuffles, atomics, which warp -- cannot change any result).  4 lanes per row, lane j holding positions 6j..6j+5;
+// each lane carries kNR rows per step (loads for all of them issued before any arithmetic).
+constexpr int kRThreads = 256;
+constexpr int kNR = 2;
+struct WarpRows {
+  int64_t r0, r1, star;
+  __device__ WarpRows(const SysView& S) {
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int64_t chunk = ((S.n_rows + nw - 1) / nw + 7) & ~(int64_t)7;
+    r0 = gw * chunk < S.n_rows ? gw * chunk : S.n_rows;
+    r1 = r0 + chunk < S.n_rows ? r0 + chunk : S.n_rows;
+    int64_t lo = 0, hi = S.n_stars;  // star of row r0: star_ptr[lo] <= r0 < star_ptr[lo + 1]
+    while (hi - lo > 1) {
+      const int64_t mid = (lo + hi) >> 1;
+      if (S.star_ptr[mid] <= r0) lo = mid;
+      else hi = mid;
+    }
+    star = lo;
   }
-  return lo;
-}
+};
 
-// value of paper slot sl of local row `row` (rows are stored lane-major: position 6j+t holds slot_of(t, j))
-__device__ __forceinline__ void row_vals(const SysView& S, int64_t row, double (&v)[kSlots]) {
-  const double* rp = S.vals + row * kSlots;
-  for (int p = 0; p < kSlots; ++p) v[slot_of(p % 6, p / 6)] = rp[p];
+__device__ __forceinline__ void load6(const SysView& S, int64_t row, int j, double (&a)[6]) {
+  const double2* p = reinterpret_cast<const double2*>(S.vals + row * kSlots + 6 * j);
+#pragma unroll
+  for (int k = 0; k < 3; ++k) {
+    const double2 t = __ldg(p + k);
+    a[2 * k] = t.x;
+    a[2 * k + 1] = t.y;
+  }
 }
 
 // ---------------------------------------------------------------------------------------------------- kernels
 // aprod1 (P&S step a): u_hat_i <- ((-alpha) * (ib * u_hat_i)) + round(EDA_s a_is * v[col_is]); beta^2 digits.
-__global__ void k_r_aprod1(SysView S, const double* __restrict__ v, double* __restrict__ u, long long* __restrict__ b2d,
-                           long long* __restrict__ cd, const DevState* __restrict__ st, int init) {
+// init: beta^2 digits of u = b only.
+__global__ void __launch_bounds__(kRThreads) k_r_aprod1(SysView S, const double* __restrict__ v,
+                                                        double* __restrict__ u, long long* __restrict__ b2d,
+                                                        long long* __restrict__ cd, const DevState* __restrict__ st,
+                                                        int init) {
   if (!init && st->halted) return;
-  const double ib = st->inv_beta, nalpha = -st->alpha;
   Eda B;
   eda_zero(B);
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < S.n_rows; i += (int64_t)gridDim.x * blockDim.x) {
-    if (init) {  // u = b: beta^2 of b
+  if (init) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < S.n_rows;
+         i += (int64_t)gridDim.x * blockDim.x)
       eda_add(B, __dmul_rn(u[i], u[i]));
-      continue;
+    eda_flush_block(B, b2d);
+    return;
+  }
+  const double ib = st->inv_beta, nalpha = -st->alpha;
+  const int lane = threadIdx.x & 31, q = lane >> 2, j = lane & 3;
+  const WarpRows R(S);
+  int64_t star = R.star;
+  for (int64_t g0 = R.r0; g0 < R.r1; g0 += 8 * kNR) {  // warp-uniform trip count
+    double a[kNR][6], g[kNR][6];
+    IdxRec rec[kNR];
+#pragma unroll
+    for (int n = 0; n < kNR; ++n) {
+      const int64_t row = g0 + 8 * n + q;
+      if (row < R.r1) {
+        load6(S, row, j, a[n]);
+        rec[n] = S.idx[row];
+      }
     }
-    double val[kSlots];
-    int64_t col[kSlots];
-    row_vals(S, i, val);
-    ic_cols(S, S.idx[i], star_of(S, i), col);
-    Eda A;
-    eda_zero(A);
-    for (int sl = 0; sl < kSlots; ++sl) {
-      if (sl == 23 && S.n_glob == 0) continue;
-      eda_add(A, __dmul_rn(val[sl], v[col[sl]]));
+#pragma unroll
+    for (int n = 0; n < kNR; ++n) {
+      const int64_t row = g0 + 8 * n + q;
+      if (row < R.r1) {
+        while (S.star_ptr[star + 1] <= row) ++star;
+#pragma unroll
+        for (int t = 0; t < 6; ++t) {
+          const int64_t c = lane_col(S, rec[n], star, t, j);
+          g[n][t] = c >= 0 ? __ldg(v + c) : 0.0;
+        }
+      }
     }
-    const double un = __dadd_rn(__dmul_rn(nalpha, __dmul_rn(ib, u[i])), eda_round_d(A.d));
-    u[i] = un;
-    eda_add(B, __dmul_rn(un, un));
+#pragma unroll
+    for (int n = 0; n < kNR; ++n) {
+      const int64_t row = g0 + 8 * n + q;
+      const bool valid = row < R.r1;
+      Eda A;
+      eda_zero(A);
+      if (valid) {
+#pragma unroll
+        for (int t = 0; t < 6; ++t) eda_add(A, __dmul_rn(a[n][t], g[n][t]));
+      }
+#pragma unroll
+      for (int k = 0; k < kL; ++k) {
+        A.d[k] += __shfl_xor_sync(0xffffffffu, A.d[k], 1);
+        A.d[k] += __shfl_xor_sync(0xffffffffu, A.d[k], 2);
+      }
+      if (valid && j == 0) {
+        const double un = __dadd_rn(__dmul_rn(nalpha, __dmul_rn(ib, u[row])), eda_round_d(A.d));
+        u[row] = un;
+        eda_add(B, __dmul_rn(un, un));
+      }
+    }
   }
   eda_flush_block(B, b2d);
-  if (init) return;
   // constraint rows: digits of every owned entry's product, one thread per chunk (chunks lie within one row)
-  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < S.n_chunks; q += (int64_t)gridDim.x * blockDim.x) {
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < S.n_chunks; c += (int64_t)gridDim.x * blockDim.x) {
     Eda A;
     eda_zero(A);
-    for (int64_t e = S.ch_beg[q]; e < S.ch_end[q]; ++e) eda_add(A, __dmul_rn(S.cval[e], v[S.ccol[e]]));
-    eda_atomic(cd + (int64_t)S.ch_row[q] * kL, A);
+    for (int64_t e = S.ch_beg[c]; e < S.ch_end[c]; ++e) eda_add(A, __dmul_rn(S.cval[e], v[S.ccol[e]]));
+    eda_atomic(cd + (int64_t)S.ch_row[c] * kL, A);
+  }
+}
+
+// aprod2 contributions: digits of a_ij * (ib * u_hat_i) into zd[q][col] (digit-major) for every column (colnorm: a_ij^2).  Astro
+// digits stay in registers per lane until the lane's star changes, global digits until the end (block-reduced);
+// attitude and instrumental digits go straight to global 64-bit integer atomics.
+__device__ __forceinline__ void flush_lane(long long* __restrict__ dst, Eda& A, int64_t stride) {
+  eda_atomic(dst, A, stride);
+  eda_zero(A);
+}
+
+__global__ void __launch_bounds__(kRThreads) k_r_aprod2(SysView S, const double* __restrict__ u,
+                                                        const double* __restrict__ uc, long long* __restrict__ zd,
+                                                        const DevState* __restrict__ st, int colnorm) {
+  if (!colnorm && (st->halted || !st->beta_pos)) return;
+  const double ib = colnorm ? 1.0 : st->inv_beta;
+  const int lane = threadIdx.x & 31, q = lane >> 2, j = lane & 3;
+  const WarpRows R(S);
+  int64_t star = R.star;
+  Eda As0, As1, G;  // astro column j (and 4 for j == 0) of `star`; global column
+  eda_zero(As0);
+  eda_zero(As1);
+  eda_zero(G);
+  for (int64_t g0 = R.r0; g0 < R.r1; g0 += 8 * kNR) {  // (no warp collectives in this loop)
+    double a[kNR][6], y[kNR];
+    IdxRec rec[kNR];
+#pragma unroll
+    for (int n = 0; n < kNR; ++n) {
+      const int64_t row = g0 + 8 * n + q;
+      if (row < R.r1) {
+        load6(S, row, j, a[n]);
+        rec[n] = S.idx[row];
+        y[n] = colnorm ? 0.0 : __ldg(u + row);
+      }
+    }
+#pragma unroll
+    for (int n = 0; n < kNR; ++n) {
+      const int64_t row = g0 + 8 * n + q;
+      if (row >= R.r1) break;
+      if (S.star_ptr[star + 1] <= row) {
+        flush_lane(zd + 5 * star + j, As0, S.n_cols);
+        if (j == 0) flush_lane(zd + 5 * star + 4, As1, S.n_cols);
+        while (S.star_ptr[star + 1] <= row) ++star;
+      }
+      const double yn = colnorm ? 0.0 : __dmul_rn(ib, y[n]);
+#pragma unroll
+      for (int t = 0; t < 6; ++t) {
+        const double term = colnorm ? __dmul_rn(a[n][t], a[n][t]) : __dmul_rn(a[n][t], yn);
+        if (t == 0) {
+          eda_add(As0, term);
+        } else if (t == 5 && j == 0) {
+          eda_add(As1, term);
+        } else if (t == 5 && j == 3) {
+          if (S.n_glob) eda_add(G, term);
+        } else {
+          eda_atomic_term(zd + lane_col(S, rec[n], star, t, j), S.n_cols, term);
+        }
+      }
+    }
+  }
+  if (R.r1 > R.r0) {
+    flush_lane(zd + 5 * star + j, As0, S.n_cols);
+    if (j == 0) flush_lane(zd + 5 * star + 4, As1, S.n_cols);
+  }
+  eda_flush_block(G, S.n_glob ? zd + S.G0 : nullptr, S.n_cols);
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < S.n_chunks; c += (int64_t)gridDim.x * blockDim.x) {
+    const double yc = colnorm ? 0.0 : __dmul_rn(ib, uc[S.ch_row[c]]);
+    for (int64_t e = S.ch_beg[c]; e < S.ch_end[c]; ++e) {
+      const double cv = S.cval[e];
+      eda_atomic_term(zd + S.ccol[e], S.n_cols, colnorm ? __dmul_rn(cv, cv) : __dmul_rn(cv, yc));
+    }
   }
 }
 
@@ -192,37 +353,6 @@ __global__ void k_r_beta(SysView S, long long* __restrict__ b2d, long long* __re
   st->inv_beta = pos ? __ddiv_rn(1.0, beta) : 1.0;
 }
 
-// aprod2 contributions: digits of a_ij * (ib * u_hat_i) into zd[col] (all columns), constraint entries likewise
-__global__ void k_r_aprod2(SysView S, const double* __restrict__ u, const double* __restrict__ uc,
-                           long long* __restrict__ zd, const DevState* __restrict__ st, int colnorm) {
-  if (!colnorm && (st->halted || !st->beta_pos)) return;
-  const double ib = colnorm ? 1.0 : st->inv_beta;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < S.n_rows; i += (int64_t)gridDim.x * blockDim.x) {
-    double val[kSlots];
-    int64_t col[kSlots];
-    row_vals(S, i, val);
-    ic_cols(S, S.idx[i], star_of(S, i), col);
-    const double y = colnorm ? 0.0 : __dmul_rn(ib, u[i]);
-    for (int sl = 0; sl < kSlots; ++sl) {
-      if (sl == 23 && S.n_glob == 0) continue;
-      Eda A;
-      eda_zero(A);
-      eda_add(A, colnorm ? __dmul_rn(val[sl], val[sl]) : __dmul_rn(val[sl], y));
-      eda_atomic(zd + col[sl] * kL, A);
-    }
-  }
-  for (int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; q < S.n_chunks; q += (int64_t)gridDim.x * blockDim.x) {
-    const double yc = colnorm ? 0.0 : __dmul_rn(ib, uc[S.ch_row[q]]);
-    for (int64_t e = S.ch_beg[q]; e < S.ch_end[q]; ++e) {
-      const double cv = S.cval[e];
-      Eda A;
-      eda_zero(A);
-      eda_add(A, colnorm ? __dmul_rn(cv, cv) : __dmul_rn(cv, yc));
-      eda_atomic(zd + S.ccol[e] * kL, A);
-    }
-  }
-}
-
 // v_j <- ((-beta) * v_j) + round(zd_j) on every column (init: v_j = 0 + round(zd_j)); alpha^2 digits; zd reset.
 // colnorm: D_j = 1/sqrt(c_j) (1 if c_j == 0) with c_j = round(zd_j).
 __global__ void k_r_vupdate(int64_t n, double* __restrict__ v, long long* __restrict__ zd, long long* __restrict__ a2d,
@@ -233,9 +363,13 @@ __global__ void k_r_vupdate(int64_t n, double* __restrict__ v, long long* __rest
   Eda A;
   eda_zero(A);
   for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x) {
-    const double z = eda_round_d(zd + c * kL);
+    long long dz[kL];
 #pragma unroll
-    for (int q = 0; q < kL; ++q) zd[c * kL + q] = 0;
+    for (int q = 0; q < kL; ++q) {
+      dz[q] = zd[q * n + c];
+      zd[q * n + c] = 0;
+    }
+    const double z = eda_round_d(dz);
     if (mode == 2) {
       v[c] = z > 0.0 ? __ddiv_rn(1.0, __dsqrt_rn(z)) : 1.0;
       continue;
@@ -392,6 +526,15 @@ __global__ void k_r_scalar_b(DevState* __restrict__ st, long long* __restrict__ 
   if (host_flag) *reinterpret_cast<volatile int32_t*>(host_flag) = st->halted | (st->itn << 1);
 }
 
+// one full wave of resident CTAs (the row partition gives every warp an equal slice)
+template <class K>
+int resident_grid(K kernel, int n_sm) {
+  int per_sm = 1;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, kRThreads, 0) != cudaSuccess || per_sm < 1)
+    per_sm = 1;
+  return n_sm * per_sm;
+}
+
 int grid_for(int64_t n) {
   int64_t b = (n + kRedThreads - 1) / kRedThreads;
   if (b < 1) b = 1;
@@ -402,27 +545,31 @@ int grid_for(int64_t n) {
 
 int64_t repro_digits_per_value() { return kL; }
 
-cudaError_t repro_iteration(const SysView& S, double* u, double* uc, const double* crhs, double* v, double* w,
+cudaError_t repro_iteration(const SysView& S, int grid, double* u, double* uc, const double* crhs, double* v, double* w,
                             double* x, double* var, long long* zd, long long* sd, DevState* st, int32_t* host_flag,
                             int init, cudaStream_t s) {
   long long* b2d = sd;       // beta^2 digits
   long long* a2d = sd + kL;  // alpha^2 digits
   long long* ddd = sd + 2 * kL;
   long long* cd = sd + 3 * kL;  // constraint row digits [n_constr][kL]
-  const int gr = grid_for(S.n_rows > S.n_chunks ? S.n_rows : S.n_chunks);
   const int gc = grid_for(S.n_cols);
+  static int g1 = 0, g2 = 0;  // per process (one device type)
+  if (!g1) {
+    g1 = resident_grid(k_r_aprod1, grid);
+    g2 = resident_grid(k_r_aprod2, grid);
+  }
   if (init) {
-    k_r_aprod1<<<gr, kRedThreads, 0, s>>>(S, v, u, b2d, cd, st, 1);
+    k_r_aprod1<<<g1, kRThreads, 0, s>>>(S, v, u, b2d, cd, st, 1);
     k_r_beta<<<1, 32, 0, s>>>(S, b2d, cd, uc, crhs, st, 1);
-    k_r_aprod2<<<gr, kRedThreads, 0, s>>>(S, u, uc, zd, st, 0);
+    k_r_aprod2<<<g2, kRThreads, 0, s>>>(S, u, uc, zd, st, 0);
     k_r_vupdate<<<gc, kRedThreads, 0, s>>>(S.n_cols, v, zd, a2d, st, 1);
     k_r_scalar_a<<<1, 32, 0, s>>>(st, a2d, 1, host_flag);
     k_r_colupdate<<<gc, kRedThreads, 0, s>>>(v, w, x, var, S.n_cols, ddd, st, 1);
     return cudaGetLastError();
   }
-  k_r_aprod1<<<gr, kRedThreads, 0, s>>>(S, v, u, b2d, cd, st, 0);
+  k_r_aprod1<<<g1, kRThreads, 0, s>>>(S, v, u, b2d, cd, st, 0);
   k_r_beta<<<1, 32, 0, s>>>(S, b2d, cd, uc, crhs, st, 0);
-  k_r_aprod2<<<gr, kRedThreads, 0, s>>>(S, u, uc, zd, st, 0);
+  k_r_aprod2<<<g2, kRThreads, 0, s>>>(S, u, uc, zd, st, 0);
   k_r_vupdate<<<gc, kRedThreads, 0, s>>>(S.n_cols, v, zd, a2d, st, 0);
   k_r_scalar_a<<<1, 32, 0, s>>>(st, a2d, 0, nullptr);
   k_r_colupdate<<<gc, kRedThreads, 0, s>>>(v, w, x, var, S.n_cols, ddd, st, 0);
@@ -430,9 +577,8 @@ cudaError_t repro_iteration(const SysView& S, double* u, double* uc, const doubl
   return cudaGetLastError();
 }
 
-cudaError_t repro_colnorm_D(const SysView& S, double* D, long long* zd, cudaStream_t s) {
-  const int gr = grid_for(S.n_rows > S.n_chunks ? S.n_rows : S.n_chunks);
-  k_r_aprod2<<<gr, kRedThreads, 0, s>>>(S, nullptr, nullptr, zd, nullptr, 1);
+cudaError_t repro_colnorm_D(const SysView& S, int grid, double* D, long long* zd, cudaStream_t s) {
+  k_r_aprod2<<<resident_grid(k_r_aprod2, grid), kRThreads, 0, s>>>(S, nullptr, nullptr, zd, nullptr, 1);
   k_r_vupdate<<<grid_for(S.n_cols), kRedThreads, 0, s>>>(S.n_cols, D, zd, nullptr, nullptr, 2);
   return cudaGetLastError();
 }
