@@ -192,9 +192,11 @@ int lsqr_get_precond(lsqr_t h, double* D);
  * order-independent digit accumulation rounded once, and every other step as one IEEE operation without FMA
  * contraction, in the order of Paige & Saunders' recurrence.  The iterates are then bit-identical run
  * to run and to the CPU oracle's repro mode, independent of scheduling; lsqr_solve_params.fused is ignored and the
- * iteration is several times slower than the default path (verification mode).  Single rank only
- * (LSQR_EINVAL when nranks > 1).  Allocates 40 B per local column of digit storage (LSQR_ENOMEM).  Invalidates a
- * previous lsqr_init; call before lsqr_precondition for a reproducible D. */
+ * iteration is several times slower than the default path (verification mode).  With nranks > 1 the digits are
+ * allreduced exactly (as pairs of exact doubles), so D, x, se and every scalar are bit-identical for ANY number of
+ * ranks and any shard map.  Allocates 40 B per local column of digit storage (+ 80 B per shared column when
+ * nranks > 1; LSQR_ENOMEM).  Invalidates a previous lsqr_init; call before lsqr_precondition for a reproducible D.
+ * Collective when nranks > 1 (only in the sense that all ranks must use the same mode). */
 int lsqr_set_reproducible(lsqr_t h, int32_t on);
 
 /* ---------------------------------------------------------------- products (hot path) */

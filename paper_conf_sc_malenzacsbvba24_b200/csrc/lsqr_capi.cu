@@ -115,6 +115,7 @@ struct lsqr_ctx {
   // NEXT-4 bitwise-reproducible mode: digit buffers (lsqr_repro.cu)
   bool repro = false;
   long long *rzd = nullptr, *rsd = nullptr;
+  double* rbuf = nullptr;  // digit allreduce staging (P > 1)
   std::string err;
 };
 
@@ -239,6 +240,45 @@ int launch_ok(lsqr_t h, cudaError_t e, const char* what) {
     if (r_ != LSQR_OK) return r_;               \
   } while (0)
 
+// ------------------------------------------------------------------------------------------------ repro mode
+// NEXT-4: allreduce of int64 digits as exact double pairs (no-op on one rank)
+int repro_allreduce(lsqr_t h, long long* src, int64_t n, int nseg, int64_t stride) {
+  if (h->nranks == 1 || n * nseg == 0) return LSQR_OK;
+  CKL(h, repro_pack(src, n, nseg, stride, h->rbuf, 0, h->s), "repro_pack");
+  CKR(allreduce(h, h->rbuf, 2 * n * nseg));
+  CKL(h, repro_pack(src, n, nseg, stride, h->rbuf, 1, h->s), "repro_unpack");
+  return LSQR_OK;
+}
+
+ReproArgs repro_args(lsqr_t h, int init) {
+  ReproArgs a;
+  a.S = h->S; a.n_sm = h->n_sm; a.init = init;
+  a.u = h->u; a.uc = h->uc; a.v = h->v; a.w = h->w; a.x = h->x; a.var = h->var; a.D = h->D; a.crhs = h->crhs;
+  a.zd = h->rzd; a.sd = h->rsd; a.st = h->st; a.host_flag = h->hflag_dev;
+  return a;
+}
+
+// One reproducible iteration (init: O-1).  P > 1: four exact digit allreduces -- [beta^2 | constraint rows] before
+// beta, the shared slice of zd before the v update, the astro alpha^2 and ddnorm digits before the scalar steps.
+int enqueue_repro(lsqr_t h, int init) {
+  const ReproArgs a = repro_args(h, init);
+  const int64_t nc = h->n_constr;
+  cudaStream_t s = h->s;
+  CKL(h, repro_step(RS_APROD1, a, s), "repro_aprod1");
+  CKR(repro_allreduce(h, repro_sd_part(h->rsd, nc, 0), 5 * (1 + nc), 1, 0));
+  CKL(h, repro_step(RS_BETA, a, s), "repro_beta");
+  CKL(h, repro_step(RS_APROD2, a, s), "repro_aprod2");
+  CKR(repro_allreduce(h, h->rzd + h->S.A0, h->n_sh, 5, h->n_loc_cols));
+  CKL(h, repro_step(RS_VUPDATE, a, s), "repro_vupdate");
+  CKR(repro_allreduce(h, repro_sd_part(h->rsd, nc, 1), 5, 1, 0));
+  CKL(h, repro_step(RS_SCALAR_A, a, s), "repro_scalar_a");
+  CKL(h, repro_step(RS_COLUPDATE, a, s), "repro_colupdate");
+  if (init) return LSQR_OK;
+  CKR(repro_allreduce(h, repro_sd_part(h->rsd, nc, 2), 5, 1, 0));
+  CKL(h, repro_step(RS_SCALAR_B, a, s), "repro_scalar_b");
+  return LSQR_OK;
+}
+
 // ------------------------------------------------------------------------------------------------ iteration
 // One LSQR iteration, all stream-ordered on h->s.  timing: optional events around the two
 // products ([0..1] aprod1, [2..3] aprod2).
@@ -247,10 +287,9 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   cudaStream_t s = h->s;
   const bool multi = h->nranks > 1;
   const bool fused = h->params.fused != 0;
-  if (h->repro) {  // NEXT-4: 7 launches, all in lsqr_repro.cu
+  if (h->repro) {  // NEXT-4: 7 launches (+ 4 x pack/unpack when P > 1), all in lsqr_repro.cu
     if (ev) cudaEventRecord(ev[0], s);
-    CKL(h, repro_iteration(S, h->grid, h->u, h->uc, h->crhs, h->v, h->w, h->x, h->var, h->rzd, h->rsd, h->st, h->hflag_dev,
-                           0, s), "repro");
+    CKR(enqueue_repro(h, 0));
     if (ev) for (int k = 1; k < 4; ++k) cudaEventRecord(ev[k], s);
     return LSQR_OK;
   }
@@ -311,7 +350,10 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   return LSQR_OK;
 }
 
-int kernels_per_iteration(lsqr_t h) { return h->repro ? 7 : (h->nranks > 1 ? 9 : (h->params.fused ? 4 : 6)); }
+int kernels_per_iteration(lsqr_t h) {
+  if (h->repro) return h->nranks > 1 ? 15 : 7;
+  return h->nranks > 1 ? 9 : (h->params.fused ? 4 : 6);
+}
 
 int build_graph(lsqr_t h) {
   if (h->gexec) {
@@ -838,7 +880,10 @@ int lsqr_precondition(lsqr_t h) {
   SysView& S = h->S;
   enter(h);
   if (h->repro) {  // NEXT-4: exact column sums of squares
-    CKL(h, repro_colnorm_D(S, h->grid, h->D, h->rzd, h->s), "colnorm_repro");
+    const ReproArgs a = repro_args(h, 0);
+    CKL(h, repro_step(RS_COLNORM, a, h->s), "colnorm_repro");
+    CKR(repro_allreduce(h, h->rzd + S.A0, h->n_sh, 5, h->n_loc_cols));
+    CKL(h, repro_step(RS_PRECOND_D, a, h->s), "precond_D_repro");
     CKL(h, launch_scale_rows(S, h->grid, h->vals, h->D, h->s), "scale_rows");
     CKL(h, launch_scale_constr(S, const_cast<double*>(S.cval), h->D, h->s), "scale_constr");
     leave(h);
@@ -873,12 +918,13 @@ int lsqr_get_precond(lsqr_t h, double* D) {
 int lsqr_set_reproducible(lsqr_t h, int32_t on) {
   GUARD(h);
   if (on != 0 && on != 1) return LSQR_EINVAL;
-  if (on && h->nranks > 1) return fail(h, LSQR_EINVAL, "reproducible mode is single-rank");
   if (on && !h->rzd) {
-    CKR(dalloc(h, &h->rzd, repro_digits_per_value() * h->n_loc_cols));
-    CKR(dalloc(h, &h->rsd, repro_digits_per_value() * (3 + h->n_constr)));
-    CKC(h, cudaMemset(h->rzd, 0, sizeof(long long) * 5 * h->n_loc_cols));
-    CKC(h, cudaMemset(h->rsd, 0, sizeof(long long) * (15 + 5 * h->n_constr)));
+    const int64_t L = repro_digits_per_value();
+    CKR(dalloc(h, &h->rzd, L * h->n_loc_cols));
+    CKR(dalloc(h, &h->rsd, repro_sd_size(h->n_constr)));
+    if (h->nranks > 1) CKR(dalloc(h, &h->rbuf, 2 * std::max<int64_t>(L * h->n_sh, repro_sd_size(h->n_constr))));
+    CKC(h, cudaMemset(h->rzd, 0, sizeof(long long) * L * h->n_loc_cols));
+    CKC(h, cudaMemset(h->rsd, 0, sizeof(long long) * repro_sd_size(h->n_constr)));
   }
   h->repro = on != 0;
   h->initialized = false;
@@ -940,9 +986,8 @@ int lsqr_init(lsqr_t h, const lsqr_solve_params* p) {
   CKL(h, launch_fill(h->zsh, h->n_sh + 8, 0.0, h->s), "fill");
   if (h->repro) {  // NEXT-4 O-1
     CKC(h, cudaMemsetAsync(h->rzd, 0, sizeof(long long) * 5 * h->n_loc_cols, h->s));
-    CKC(h, cudaMemsetAsync(h->rsd, 0, sizeof(long long) * (15 + 5 * h->n_constr), h->s));
-    CKL(h, repro_iteration(S, h->grid, h->u, h->uc, h->crhs, h->v, h->w, h->x, h->var, h->rzd, h->rsd, h->st, h->hflag_dev,
-                           1, h->s), "repro_init");
+    CKC(h, cudaMemsetAsync(h->rsd, 0, sizeof(long long) * repro_sd_size(h->n_constr), h->s));
+    CKR(enqueue_repro(h, 1));
     h->b_valid = false;
     h->initialized = true;
     if (p->use_graph) CKR(build_graph(h));

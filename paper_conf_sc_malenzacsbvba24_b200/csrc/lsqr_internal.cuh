@@ -171,15 +171,29 @@ cudaError_t launch_finalize(const double* x, const double* var, const double* D,
                             double se_t, double* x_out, double* se_out, cudaStream_t s);
 cudaError_t launch_fill(double* p, int64_t n, double v, cudaStream_t s);
 
-// NEXT-4 bitwise-reproducible mode (lsqr_repro.cu, docs/REPRO.md).  Digit buffers: zd [5][n_cols] (digit-major; zeroed;
-// left zeroed), sd [15 + 5 n_constr] (beta^2 | alpha^2 | ddnorm | constraint rows; zeroed, left zeroed).  u / uc hold
-// u_hat (unnormalised) like the default path; st->inv_beta normalises.  grid: the persistent row-kernel grid
-// (kThreads per CTA) that SysView::warp_star partitions.
+// NEXT-4 bitwise-reproducible mode (lsqr_repro.cu, docs/REPRO.md).  Digit buffers (int64, zeroed; every step leaves
+// what it consumed zeroed): zd [5][n_cols] digit-major column accumulator; sd [repro_sd_size(n_constr)] =
+// [beta^2 (5) | constraint rows (5 n_constr) | alpha^2 astro (5) | alpha^2 shared (5) | ddnorm astro (5) |
+// ddnorm shared (5)].  The astro parts are rank-local (allreduced when P > 1), the shared parts are computed
+// identically on every rank.  u / uc hold u_hat (unnormalised) like the default path; st->inv_beta normalises.
+enum { RS_APROD1, RS_BETA, RS_APROD2, RS_VUPDATE, RS_SCALAR_A, RS_COLUPDATE, RS_SCALAR_B, RS_COLNORM, RS_PRECOND_D };
+struct ReproArgs {
+  SysView S;
+  int n_sm, init;
+  double *u, *uc, *v, *w, *x, *var, *D;
+  const double* crhs;
+  long long *zd, *sd;
+  DevState* st;
+  int32_t* host_flag;
+};
 int64_t repro_digits_per_value();
-cudaError_t repro_iteration(const SysView& S, int grid, double* u, double* uc, const double* crhs, double* v, double* w,
-                            double* x, double* var, long long* zd, long long* sd, DevState* st, int32_t* host_flag,
-                            int init, cudaStream_t s);
-// D_j = 1/sqrt(round(EDA sum a_ij^2)) (1 if 0) over the local rows and owned constraint entries (single rank)
-cudaError_t repro_colnorm_D(const SysView& S, int grid, double* D, long long* zd, cudaStream_t s);
+int64_t repro_sd_size(int64_t n_constr);
+// part 0: [beta^2 | constraint rows] (5 + 5 n_constr contiguous), 1: alpha^2 astro (5), 2: ddnorm astro (5)
+long long* repro_sd_part(long long* sd, int64_t n_constr, int part);
+cudaError_t repro_step(int step, const ReproArgs& a, cudaStream_t s);
+// int64 <-> exact double pairs for the allreduce: nseg segments of n values, segment stride `stride` (in values);
+// buf holds 2 n nseg doubles
+cudaError_t repro_pack(const long long* src, int64_t n, int nseg, int64_t stride, double* buf, int unpack,
+                       cudaStream_t s);
 
 }  // namespace lsqr

@@ -353,15 +353,18 @@ __global__ void k_r_beta(SysView S, long long* __restrict__ b2d, long long* __re
   st->inv_beta = pos ? __ddiv_rn(1.0, beta) : 1.0;
 }
 
-// v_j <- ((-beta) * v_j) + round(zd_j) on every column (init: v_j = 0 + round(zd_j)); alpha^2 digits; zd reset.
-// colnorm: D_j = 1/sqrt(c_j) (1 if c_j == 0) with c_j = round(zd_j).
-__global__ void k_r_vupdate(int64_t n, double* __restrict__ v, long long* __restrict__ zd, long long* __restrict__ a2d,
-                            const DevState* __restrict__ st, int mode) {  // mode 0 LSQR, 1 init, 2 colnorm -> D
+// v_j <- ((-beta) * v_j) + round(zd_j) on every column (init: v_j = 0 + round(zd_j)); alpha^2 digits split into the
+// astro part (columns < A0, rank-local: allreduced when P > 1) and the shared part (replicated on every rank: never
+// reduced); zd reset.  mode 2 (colnorm): D_j = 1/sqrt(c_j) (1 if c_j == 0) with c_j = round(zd_j).
+__global__ void k_r_vupdate(int64_t n, int64_t A0, double* __restrict__ v, long long* __restrict__ zd,
+                            long long* __restrict__ a2d, long long* __restrict__ a2s, const DevState* __restrict__ st,
+                            int mode) {  // mode 0 LSQR, 1 init, 2 colnorm -> D
   if (mode == 0 && (st->halted || !st->beta_pos)) return;
   if (mode == 1 && !st->beta_pos) return;
   const double nbeta = mode == 2 ? 0.0 : -st->beta;
-  Eda A;
-  eda_zero(A);
+  Eda Aa, As;
+  eda_zero(Aa);
+  eda_zero(As);
   for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < n; c += (int64_t)gridDim.x * blockDim.x) {
     long long dz[kL];
 #pragma unroll
@@ -376,13 +379,17 @@ __global__ void k_r_vupdate(int64_t n, double* __restrict__ v, long long* __rest
     }
     const double vn = mode == 1 ? __dadd_rn(v[c], z) : __dadd_rn(__dmul_rn(nbeta, v[c]), z);
     v[c] = vn;
-    eda_add(A, __dmul_rn(vn, vn));
+    eda_add(c < A0 ? Aa : As, __dmul_rn(vn, vn));
   }
-  if (mode != 2) eda_flush_block(A, a2d);
+  if (mode != 2) {
+    eda_flush_block(Aa, a2d);
+    eda_flush_block(As, a2s);
+  }
 }
 
 // P&S steps b (alpha), c, d (rotation): t1, t2, t3 -- one thread
-__global__ void k_r_scalar_a(DevState* __restrict__ st, long long* __restrict__ a2d, int init, int32_t* __restrict__ host_flag) {
+__global__ void k_r_scalar_a(DevState* __restrict__ st, long long* __restrict__ a2d, long long* __restrict__ a2s,
+                             int init, int32_t* __restrict__ host_flag) {
   if (threadIdx.x != 0 || blockIdx.x != 0) return;
   if (!init && st->halted) {
     st->col_enable = 0;
@@ -391,13 +398,15 @@ __global__ void k_r_scalar_a(DevState* __restrict__ st, long long* __restrict__ 
   const int bp = st->beta_pos;
   double alpha = st->alpha;
   if (bp) {
-    alpha = __dsqrt_rn(eda_round_d(a2d));
+    long long a2[kL];
+    for (int q = 0; q < kL; ++q) a2[q] = a2d[q] + a2s[q];
+    alpha = __dsqrt_rn(eda_round_d(a2));
     st->inv_alpha = alpha > 0.0 ? __ddiv_rn(1.0, alpha) : 1.0;
     st->v_pending = 1;
   } else {
     st->v_pending = 0;
   }
-  for (int q = 0; q < kL; ++q) a2d[q] = 0;
+  for (int q = 0; q < kL; ++q) a2d[q] = a2s[q] = 0;
   st->alpha = alpha;
   st->col_enable = 1;
   if (init) {  // O-1/O-2
@@ -442,13 +451,14 @@ __global__ void k_r_scalar_a(DevState* __restrict__ st, long long* __restrict__ 
 
 // O-3e: v <- (1/alpha) v (if pending); d = t3 w; var += d*d; x += t1 w; w = v + t2 w; ddnorm digits
 __global__ void k_r_colupdate(double* __restrict__ v, double* __restrict__ w, double* __restrict__ x,
-                              double* __restrict__ var, int64_t n, long long* __restrict__ ddd,
-                              const DevState* __restrict__ st, int init) {
+                              double* __restrict__ var, int64_t n, int64_t A0, long long* __restrict__ ddd,
+                              long long* __restrict__ dds, const DevState* __restrict__ st, int init) {
   if (!st->col_enable) return;
   const double ia = st->inv_alpha, t1 = st->t1, t2 = st->t2, t3 = st->t3;
   const int vp = st->v_pending && st->alpha > 0.0;
-  Eda A;
-  eda_zero(A);
+  Eda Aa, As;  // ddnorm digits: astro (rank-local) / shared (replicated)
+  eda_zero(Aa);
+  eda_zero(As);
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     const double vi = vp ? __dmul_rn(ia, v[i]) : v[i];
     v[i] = vi;
@@ -460,22 +470,30 @@ __global__ void k_r_colupdate(double* __restrict__ v, double* __restrict__ w, do
     const double dk = __dmul_rn(t3, wi);
     const double d2 = __dmul_rn(dk, dk);
     var[i] = __dadd_rn(var[i], d2);
-    eda_add(A, d2);
+    eda_add(i < A0 ? Aa : As, d2);
     x[i] = __dadd_rn(x[i], __dmul_rn(t1, wi));
     w[i] = __dadd_rn(vi, __dmul_rn(t2, wi));
   }
-  if (!init) eda_flush_block(A, ddd);
+  if (!init) {
+    eda_flush_block(Aa, ddd);
+    eda_flush_block(As, dds);
+  }
 }
 
 // O-3f-j after the column update (ddnorm needed by acond) -- one thread
-__global__ void k_r_scalar_b(DevState* __restrict__ st, long long* __restrict__ ddd, int32_t* __restrict__ host_flag) {
+__global__ void k_r_scalar_b(DevState* __restrict__ st, long long* __restrict__ ddd, long long* __restrict__ dds,
+                             int32_t* __restrict__ host_flag) {
   if (threadIdx.x != 0 || blockIdx.x != 0) return;
   if (st->halted || !st->col_enable) return;
   const double eps = 0x1p-52;
   const double rho = st->r_rho, theta = st->r_theta, phi = st->r_phi, sn = st->r_sn, psi = st->rn_tmp;
   const double tau = __dmul_rn(sn, phi);
-  const double ddnorm = __dadd_rn(st->ddnorm, eda_round_d(ddd));
-  for (int q = 0; q < kL; ++q) ddd[q] = 0;
+  long long dd[kL];
+  for (int q = 0; q < kL; ++q) {
+    dd[q] = ddd[q] + dds[q];
+    ddd[q] = dds[q] = 0;
+  }
+  const double ddnorm = __dadd_rn(st->ddnorm, eda_round_d(dd));
   // f.
   const double delta = __dmul_rn(st->sn2, rho), gambar = __dmul_rn(-st->cs2, rho);
   const double rhs = __dadd_rn(phi, -__dmul_rn(delta, st->z));
@@ -526,6 +544,28 @@ __global__ void k_r_scalar_b(DevState* __restrict__ st, long long* __restrict__ 
   if (host_flag) *reinterpret_cast<volatile int32_t*>(host_flag) = st->halted | (st->itn << 1);
 }
 
+// int64 digits <-> pairs of exact doubles (signed high 32 bits, unsigned low 32 bits) for the FP64 SUM allreduce:
+// every partial sum of P such halves is an integer below 2^53 in magnitude, hence exact in any order.
+__global__ void k_r_pack(const long long* __restrict__ src, int64_t n, int nseg, int64_t stride,
+                         double* __restrict__ buf) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n * nseg; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t sg = i / n, o = i - sg * n;
+    const long long v = src[sg * stride + o];
+    buf[2 * i] = (double)(v >> 32);
+    buf[2 * i + 1] = (double)(v & 0xffffffffll);
+  }
+}
+
+__global__ void k_r_unpack(const double* __restrict__ buf, int64_t n, int nseg, int64_t stride,
+                           long long* __restrict__ dst) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n * nseg; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t sg = i / n, o = i - sg * n;
+    const unsigned long long hi = (unsigned long long)(long long)buf[2 * i];
+    const unsigned long long lo = (unsigned long long)(long long)buf[2 * i + 1];
+    dst[sg * stride + o] = (long long)((hi << 32) + lo);  // two's-complement wrap-around = the int64 sum
+  }
+}
+
 // one full wave of resident CTAs (the row partition gives every warp an equal slice)
 template <class K>
 int resident_grid(K kernel, int n_sm) {
@@ -541,45 +581,60 @@ int grid_for(int64_t n) {
   return (int)(b < 148 * 8 ? b : 148 * 8);
 }
 
+struct SdView {  // layout of the scalar digit buffer (see lsqr_internal.cuh)
+  long long *b2d, *cd, *a2d, *a2s, *ddd, *dds;
+  SdView(long long* sd, int64_t nc) {
+    b2d = sd;
+    cd = sd + kL;
+    a2d = cd + kL * nc;
+    a2s = a2d + kL;
+    ddd = a2s + kL;
+    dds = ddd + kL;
+  }
+};
+
 }  // namespace
 
 int64_t repro_digits_per_value() { return kL; }
+int64_t repro_sd_size(int64_t n_constr) { return kL * (5 + n_constr); }
+long long* repro_sd_part(long long* sd, int64_t n_constr, int part) {
+  const SdView V(sd, n_constr);
+  return part == 0 ? V.b2d : (part == 1 ? V.a2d : V.ddd);
+}
 
-cudaError_t repro_iteration(const SysView& S, int grid, double* u, double* uc, const double* crhs, double* v, double* w,
-                            double* x, double* var, long long* zd, long long* sd, DevState* st, int32_t* host_flag,
-                            int init, cudaStream_t s) {
-  long long* b2d = sd;       // beta^2 digits
-  long long* a2d = sd + kL;  // alpha^2 digits
-  long long* ddd = sd + 2 * kL;
-  long long* cd = sd + 3 * kL;  // constraint row digits [n_constr][kL]
-  const int gc = grid_for(S.n_cols);
+cudaError_t repro_step(int step, const ReproArgs& a, cudaStream_t s) {
+  const SysView& S = a.S;
+  const SdView V(a.sd, S.n_constr);
   static int g1 = 0, g2 = 0;  // per process (one device type)
   if (!g1) {
-    g1 = resident_grid(k_r_aprod1, grid);
-    g2 = resident_grid(k_r_aprod2, grid);
+    g1 = resident_grid(k_r_aprod1, a.n_sm);
+    g2 = resident_grid(k_r_aprod2, a.n_sm);
   }
-  if (init) {
-    k_r_aprod1<<<g1, kRThreads, 0, s>>>(S, v, u, b2d, cd, st, 1);
-    k_r_beta<<<1, 32, 0, s>>>(S, b2d, cd, uc, crhs, st, 1);
-    k_r_aprod2<<<g2, kRThreads, 0, s>>>(S, u, uc, zd, st, 0);
-    k_r_vupdate<<<gc, kRedThreads, 0, s>>>(S.n_cols, v, zd, a2d, st, 1);
-    k_r_scalar_a<<<1, 32, 0, s>>>(st, a2d, 1, host_flag);
-    k_r_colupdate<<<gc, kRedThreads, 0, s>>>(v, w, x, var, S.n_cols, ddd, st, 1);
-    return cudaGetLastError();
+  const int gc = grid_for(S.n_cols);
+  switch (step) {
+    case RS_APROD1: k_r_aprod1<<<g1, kRThreads, 0, s>>>(S, a.v, a.u, V.b2d, V.cd, a.st, a.init); break;
+    case RS_BETA: k_r_beta<<<1, 32, 0, s>>>(S, V.b2d, V.cd, a.uc, a.crhs, a.st, a.init); break;
+    case RS_APROD2: k_r_aprod2<<<g2, kRThreads, 0, s>>>(S, a.u, a.uc, a.zd, a.st, 0); break;
+    case RS_VUPDATE: k_r_vupdate<<<gc, kRedThreads, 0, s>>>(S.n_cols, S.A0, a.v, a.zd, V.a2d, V.a2s, a.st, a.init); break;
+    case RS_SCALAR_A: k_r_scalar_a<<<1, 32, 0, s>>>(a.st, V.a2d, V.a2s, a.init, a.init ? a.host_flag : nullptr); break;
+    case RS_COLUPDATE:
+      k_r_colupdate<<<gc, kRedThreads, 0, s>>>(a.v, a.w, a.x, a.var, S.n_cols, S.A0, V.ddd, V.dds, a.st, a.init);
+      break;
+    case RS_SCALAR_B: k_r_scalar_b<<<1, 32, 0, s>>>(a.st, V.ddd, V.dds, a.host_flag); break;
+    case RS_COLNORM: k_r_aprod2<<<g2, kRThreads, 0, s>>>(S, nullptr, nullptr, a.zd, nullptr, 1); break;
+    case RS_PRECOND_D:
+      k_r_vupdate<<<gc, kRedThreads, 0, s>>>(S.n_cols, S.A0, a.D, a.zd, nullptr, nullptr, nullptr, 2);
+      break;
+    default: return cudaErrorInvalidValue;
   }
-  k_r_aprod1<<<g1, kRThreads, 0, s>>>(S, v, u, b2d, cd, st, 0);
-  k_r_beta<<<1, 32, 0, s>>>(S, b2d, cd, uc, crhs, st, 0);
-  k_r_aprod2<<<g2, kRThreads, 0, s>>>(S, u, uc, zd, st, 0);
-  k_r_vupdate<<<gc, kRedThreads, 0, s>>>(S.n_cols, v, zd, a2d, st, 0);
-  k_r_scalar_a<<<1, 32, 0, s>>>(st, a2d, 0, nullptr);
-  k_r_colupdate<<<gc, kRedThreads, 0, s>>>(v, w, x, var, S.n_cols, ddd, st, 0);
-  k_r_scalar_b<<<1, 32, 0, s>>>(st, ddd, host_flag);
   return cudaGetLastError();
 }
 
-cudaError_t repro_colnorm_D(const SysView& S, int grid, double* D, long long* zd, cudaStream_t s) {
-  k_r_aprod2<<<resident_grid(k_r_aprod2, grid), kRThreads, 0, s>>>(S, nullptr, nullptr, zd, nullptr, 1);
-  k_r_vupdate<<<grid_for(S.n_cols), kRedThreads, 0, s>>>(S.n_cols, D, zd, nullptr, nullptr, 2);
+cudaError_t repro_pack(const long long* src, int64_t n, int nseg, int64_t stride, double* buf, int unpack,
+                       cudaStream_t s) {
+  if (n * nseg == 0) return cudaSuccess;
+  if (unpack) k_r_unpack<<<grid_for(n * nseg), kRedThreads, 0, s>>>(buf, n, nseg, stride, const_cast<long long*>(src));
+  else k_r_pack<<<grid_for(n * nseg), kRedThreads, 0, s>>>(src, n, nseg, stride, buf);
   return cudaGetLastError();
 }
 

@@ -173,3 +173,66 @@ def test_gpu_two_rank_lsqr_matches_single_rank(cuda_device, fused):
         assert np.allclose(xx[:A0l], x21[5 * sb:5 * se], rtol=1e-12, atol=1e-12)
         assert np.allclose(xx[A0l:], x21[A0:], rtol=1e-12, atol=1e-12)
     s.close()
+
+
+# ------------------------------------------------------------------------------------------------ GPU, repro mode
+def _gpu_repro_worker(rank, world, port, q, itn):
+    try:
+        import sys
+        sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+        import torch
+        import paper_conf_sc_malenzacsbvba24_b200 as avu
+        _init(rank, world, port)
+        torch.cuda.set_device(0)
+        w = W.C1C.replace(jitter_pct=50)
+        s = avu.Solver.synthetic(w, rank=rank, nranks=world, comm="callback")
+        s.set_reproducible(True)
+        s.precondition()
+        D = s.get_precond()
+        out = s.solve(itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=False)
+        q.put((rank, s.star_begin, s.star_end, out["x"], out["se"], out["itn"], out["r1norm"], out["acond"], D))
+        s.close()
+        import torch.distributed as dist
+        dist.destroy_process_group()
+    except Exception:
+        import traceback
+        q.put(("error", traceback.format_exc()))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("P", [2, 3])
+def test_gpu_repro_bitwise_across_rank_counts(cuda_device, P):
+    """NEXT-4 across ranks: the digit allreduces are exact, so D, x, sigma and the norm estimates of a P-rank
+    reproducible solve are BIT-identical to the 1-rank reproducible solve and to the oracle's repro mode -- after
+    40 iterations, long before convergence (where the default mode differs already at k ~ 10)."""
+    import oracle
+    import paper_conf_sc_malenzacsbvba24_b200 as avu
+    itn = 40
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_gpu_repro_worker, args=(r, P, port, q, itn)) for r in range(P)]
+    for p in ps:
+        p.start()
+    outs = [q.get(timeout=600) for _ in range(P)]
+    for p in ps:
+        p.join(60)
+    for o in outs:
+        assert o[0] != "error", o[1]
+    w = W.C1C.replace(jitter_pct=50)
+    s = avu.Solver.synthetic(w)
+    s.set_reproducible(True)
+    s.precondition()
+    D1 = s.get_precond()
+    ref = s.solve(itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True)
+    s.close()
+    ro = oracle.solve_system(oracle.System(w), atol=0, btol=0, conlim=0, itn_limit=itn, fixed_count=True, repro=True)
+    same = lambda a, b: np.array_equal(np.ascontiguousarray(a).view(np.uint64), np.ascontiguousarray(b).view(np.uint64))
+    assert same(ref["x"], ro["x"]) and same(ref["se"], ro["se"])
+    A0 = 5 * w.n_stars
+    for (rank, sb, se, x, sev, it, r1, ac, D) in outs:
+        A0l = 5 * (se - sb)
+        assert it == itn and r1 == ref["r1norm"] and ac == ref["acond"]
+        assert same(D[:A0l], D1[5 * sb:5 * se]) and same(D[A0l:], D1[A0:])
+        assert same(x[:A0l], ref["x"][5 * sb:5 * se]) and same(x[A0l:], ref["x"][A0:])
+        assert same(sev[:A0l], ref["se"][5 * sb:5 * se]) and same(sev[A0l:], ref["se"][A0:])
