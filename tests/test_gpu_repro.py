@@ -123,10 +123,3 @@ def test_repro_converges_like_default(avu):
     b = s.solve(**kw)
     s.close()
     assert np.linalg.norm(a["x"] - b["x"]) <= 1e-9 * np.linalg.norm(b["x"])
-
-
-def test_repro_rejects_multirank(avu):
-    s = avu.Solver.synthetic(W.C1C, rank=0, nranks=2, comm="callback", allreduce=lambda *a: 1)
-    with pytest.raises(avu.LsqrError):
-        s.set_reproducible(True)
-    s.close()
