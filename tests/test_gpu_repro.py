@@ -123,3 +123,53 @@ def test_repro_converges_like_default(avu):
     b = s.solve(**kw)
     s.close()
     assert np.linalg.norm(a["x"] - b["x"]) <= 1e-9 * np.linalg.norm(b["x"])
+
+
+def _empty_star_system():
+    """micro system whose stars 10, 11, 30, 49 have no observations (their columns are exactly zero)."""
+    import ctypes
+    w = W.micro(n_stars=50, obs=12, n_ext=6, seed=17)
+    counts = oracle.star_counts(w)
+    counts[[10, 11, 30, 49]] = 0
+    counts[0] += w.n_obs - counts.sum()
+    S = oracle.System(w, generate=False)
+    S.counts, S.row_ptr = counts, oracle.row_ptr(counts)
+    n = int(counts.sum())
+    S.n_rows, S.row_begin, S.row_end, S.star_begin, S.star_end = n, 0, n, 0, w.n_stars
+    S.vals = np.zeros((n, 24)); S.mA = np.zeros(n, dtype=np.int64); S.mT = np.zeros(n, dtype=np.int64)
+    S.iC = np.zeros((n, 6), dtype=np.int64); S.b = np.zeros(n)
+    L = oracle.lib()
+    P = lambda a: a.ctypes.data_as(ctypes.c_void_p)
+    L.orc_generate(w.seed, w.n_stars, w.n_att, w.n_instr, w.n_glob, P(S.row_ptr), 0, w.n_stars, P(S.vals), P(S.mA),
+                   P(S.mT), P(S.iC))
+    L.orc_generate_b(w.seed, 0, 0.0, w.n_stars, w.n_att, w.n_instr, w.n_glob, P(S.row_ptr), 0, w.n_stars, P(S.vals),
+                     P(S.mA), P(S.mT), P(S.iC), P(np.zeros(1)), P(S.b))
+    S._mk_struct()
+    return w, counts, S
+
+
+@pytest.mark.parametrize("case", ["damped", "empty_stars"])
+def test_repro_edge_cases_bitwise(avu, case):
+    """Damped solve (the damping rotation branch of the scalar recurrence) and stars without observations (zero
+    columns, D = 1): x, sigma and the norm estimates bit-identical to the oracle's repro mode."""
+    if case == "damped":
+        w, counts, damp = W.micro(n_stars=30, obs=25, seed=11, n_ext=5), None, 0.37
+        S = oracle.System(w)
+    else:
+        (w, counts, S), damp = _empty_star_system(), 0.0
+    host = {k: getattr(S, k).copy() for k in ("vals", "mA", "mT", "iC", "b", "c_ptr", "c_col", "c_val")}
+    ro = oracle.solve_system(S, damp=damp, atol=0, btol=0, conlim=0, itn_limit=80, fixed_count=True, repro=True)
+    if counts is None:
+        s = avu.Solver.synthetic(w)
+    else:
+        s = avu.Solver(w.n_stars, w.n_obs, w.n_att, w.n_instr, w.n_glob, obs_per_star=counts,
+                       constraints=(host["c_ptr"], host["c_col"], host["c_val"]))
+        s.set_system(host["vals"], host["mA"], host["mT"], host["iC"], host["b"])
+    s.set_reproducible(True)
+    s.precondition()
+    out = s.solve(damp=damp, atol=0, btol=0, conlim=0, itn_limit=80, fixed_count=True)
+    s.close()
+    assert same(out["x"], ro["x"]), first_diff(out["x"], ro["x"])
+    assert same(out["se"], ro["se"])
+    for k in ("r1norm", "r2norm", "anorm", "acond", "arnorm", "xnorm"):
+        assert same(out[k], ro[k]), k
