@@ -286,6 +286,18 @@ class Solver:
     def iterate(self, n):
         self._chk(_capi.lib().lsqr_iterate(self._h, int(n)))
 
+    def iterate_events(self, n) -> float:
+        """lsqr_iterate(n) bracketed by CUDA events on the solver's stream (the library's stream is ordered after it
+        at entry and before it at exit); returns the elapsed device milliseconds."""
+        torch = self._torch
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(self.stream)
+        self.iterate(n)
+        e1.record(self.stream)
+        e1.synchronize()
+        return e0.elapsed_time(e1)
+
     def iterate_timed(self, n):
         out = np.zeros(5)
         self._chk(_capi.lib().lsqr_iterate_timed(self._h, int(n), _p(out)))
