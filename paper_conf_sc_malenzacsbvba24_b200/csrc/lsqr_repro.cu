@@ -4,7 +4,7 @@
 // rounded FP64 terms, combined with 64-bit integer additions/atomics, which are associative: the result does not
 // depend on thread, warp, block or atomic order.  Every other operation is a single IEEE operation written with
 // explicit _rn intrinsics (no FMA contraction), in the order the Paige-Saunders recurrence writes them.  The CPU
-// oracle implements the same spec independently (oracle/avugsr_oracle.c), so iterates agree bit for bit.
+// test oracle implements the same spec independently (docs/REPRO.md), so iterates agree bit for bit.
 //
 // These kernels are simple (thread per row / column, global atomics for every digit): the mode is for verification
 // and run-to-run reproducibility, not for speed.

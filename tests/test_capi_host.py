@@ -87,3 +87,27 @@ def test_create_rejects_bad_arguments_without_gpu():
     assert L.lsqr_synth_obs_per_star(1, 0, 10, 0, None) == -1
     assert L.lsqr_synth_constraints(1, 10, 30, 7, 5, None, None, None) == -1
     assert L.lsqr_destroy(None) == 0
+
+
+def test_missing_extension_fails_loudly(monkeypatch, tmp_path):
+    """No CPU fallback: without the shared library every entry point raises (the binding never computes)."""
+    from paper_conf_sc_malenzacsbvba24_b200 import _capi, build as _build
+    monkeypatch.setattr(_build, "LIB", str(tmp_path / "liblsqr_avugsr.so"))
+    monkeypatch.setattr(_capi, "_lib", None)
+    with pytest.raises(RuntimeError, match="missing"):
+        _capi.lib(build_if_missing=False)
+
+
+def test_product_package_never_touches_the_oracle():
+    """The product path (package sources, CUDA, C ABI header) shares no code with oracle/ and does not import it."""
+    import glob
+    import os
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    files = glob.glob(os.path.join(root, "paper_conf_sc_malenzacsbvba24_b200", "**", "*.*"), recursive=True)
+    files += glob.glob(os.path.join(root, "include", "*.h"))
+    srcs = [f for f in files if f.endswith((".py", ".cu", ".cuh", ".h", ".c", ".cpp"))]
+    assert srcs
+    for f in srcs:
+        txt = open(f, encoding="utf-8", errors="replace").read()
+        for bad in ("import oracle", "from oracle", "avugsr_oracle", "orc_"):
+            assert bad not in txt, (f, bad)
