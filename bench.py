@@ -150,6 +150,9 @@ def _cpu_model():
 
 
 def variant_name(args):
+    if getattr(args, "force_collectives", False):
+        base = "fused single pass" if getattr(args, "fused", False) else "two-pass"
+        return base + " via the multi-rank path (forced 1-rank NCCL collectives)"
     if getattr(args, "repro", False):
         return "bitwise-reproducible (SURVEY 8(f) NEXT-4; exact digit reductions, verification mode)"
     return "fused single pass" if getattr(args, "fused", False) else "two-pass"
@@ -281,7 +284,7 @@ def run_ours(args):
     # lsqr_solve runs them), CUDA events on the library stream around the K iterations only.
     # pass 2 (kernel roofline): K more iterations through lsqr_iterate_timed, CUDA events around every kernel launch
     # (those events cost ~7 % of a C2 step, which is why they are not in pass 1).
-    s = avu.Solver.synthetic(w, rank=rank, nranks=world, **comm_kw())
+    s = avu.Solver.synthetic(w, rank=rank, nranks=world, force_collectives=args.force_collectives, **comm_kw())
     if args.repro:
         s.set_reproducible(True)
     t0 = time.perf_counter()
@@ -382,6 +385,9 @@ def main():
     ap.add_argument("--comm", default="nccl", choices=["nccl", "gloo-callback"],
                     help="multi-rank communicator (gloo-callback: test mode through the library's host callback)")
     ap.add_argument("--same-device", action="store_true", help="test mode: every rank on cuda:0")
+    ap.add_argument("--force-collectives", action="store_true",
+                    help="diagnostic: run the multi-rank algorithm and its NCCL collectives on a 1-rank communicator "
+                         "(measures the P > 1 code path's cost without a network)")
     args = ap.parse_args()
     if args.warmup < 3:
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)

@@ -74,8 +74,13 @@ typedef struct {
   lsqr_alloc_fn alloc;     /* nullable */
   lsqr_free_fn free;       /* nullable (must be set iff alloc is) */
   void* alloc_user;
-  lsqr_allreduce_fn allreduce; /* required iff nranks > 1 and comm_kind == LSQR_COMM_CALLBACK */
+  lsqr_allreduce_fn allreduce; /* required iff nranks > 1 (or force_collectives) and comm_kind == LSQR_COMM_CALLBACK */
   void* allreduce_user;
+  int32_t force_collectives; /* test hook: 1 = run the multi-rank algorithm and its collectives even when nranks == 1
+                                (NCCL: a 1-rank communicator with an internally generated id, nccl_id may be NULL;
+                                callback: the callback is called).  Results equal the nranks == 1 path up to rounding
+                                (bit-identical in the reproducible mode).  0 = normal. */
+  int32_t pad_;
 } lsqr_env;
 
 /* Constraint equations: extra sparse rows appended after the observations (content not

@@ -102,7 +102,7 @@ class Solver:
 
     def __init__(self, n_stars, n_obs, n_att, n_instr, n_glob=1, obs_per_star=None, constraints=None, rank=0,
                  nranks=1, device=None, comm="nccl", nccl_id=None, allreduce=None, stream=None,
-                 torch_alloc=True):
+                 torch_alloc=True, force_collectives=False):
         import torch
         self._torch = torch
         L = _capi.lib()
@@ -114,6 +114,7 @@ class Solver:
         env = _capi.Env()
         env.rank, env.nranks, env.device = rank, nranks, self.device
         env.comm_kind = 1 if comm == "callback" else 0
+        env.force_collectives = int(bool(force_collectives))  # test hook (lsqr_env.force_collectives)
         if nranks > 1 and env.comm_kind == 0:
             if nccl_id is None:
                 raise ValueError("nccl_id required for nranks > 1 with NCCL")
@@ -139,7 +140,7 @@ class Solver:
             fa, ff = _capi.ALLOC_FN(_alloc), _capi.FREE_FN(_free)
             self._keep += [fa, ff]
             env.alloc, env.free = fa, ff
-        if env.comm_kind == 1 and nranks > 1:
+        if env.comm_kind == 1 and (nranks > 1 or force_collectives):
             cb = _capi.ALLREDUCE_FN(allreduce or gloo_allreduce_callback())
             self._keep.append(cb)
             env.allreduce = cb

@@ -29,7 +29,7 @@ ALLREDUCE_FN = C.CFUNCTYPE(C.c_int, vp, i64, u64, vp)
 class Env(C.Structure):
     _fields_ = [("rank", i32), ("nranks", i32), ("device", i32), ("comm_kind", i32), ("nccl_id", vp),
                 ("stream", u64), ("alloc", ALLOC_FN), ("free", FREE_FN), ("alloc_user", vp),
-                ("allreduce", ALLREDUCE_FN), ("allreduce_user", vp)]
+                ("allreduce", ALLREDUCE_FN), ("allreduce_user", vp), ("force_collectives", i32), ("pad_", i32)]
 
 
 class Constraints(C.Structure):

@@ -74,6 +74,7 @@ struct lsqr_ctx {
   int32_t n_glob = 0;
   // rank
   int32_t rank = 0, nranks = 1, device = 0, comm_kind = 0;
+  bool multi = false;  // multi-rank algorithm + collectives (nranks > 1, or env->force_collectives)
   int64_t star_begin = 0, star_end = 0, row_begin = 0, row_end = 0;
   int64_t n_loc_stars = 0, n_loc_rows = 0, n_sh = 0, n_loc_cols = 0, n_constr = 0;
   std::vector<int64_t> counts;       // obs per star (global)
@@ -180,7 +181,7 @@ void leave(lsqr_t h) {
 
 // in-place SUM allreduce of count doubles on the library stream (no-op on one rank)
 int allreduce(lsqr_t h, double* buf, int64_t count) {
-  if (h->nranks == 1 || count == 0) return LSQR_OK;
+  if (!h->multi || count == 0) return LSQR_OK;
   if (h->comm_kind == LSQR_COMM_NCCL) {
     ncclResult_t r = g_nccl.AllReduce(buf, buf, (size_t)count, ncclFloat64, ncclSum, h->nccl, h->s);
     if (r != ncclSuccess)
@@ -243,7 +244,7 @@ int launch_ok(lsqr_t h, cudaError_t e, const char* what) {
 // ------------------------------------------------------------------------------------------------ repro mode
 // NEXT-4: allreduce of int64 digits as exact double pairs (no-op on one rank)
 int repro_allreduce(lsqr_t h, long long* src, int64_t n, int nseg, int64_t stride) {
-  if (h->nranks == 1 || n * nseg == 0) return LSQR_OK;
+  if (!h->multi || n * nseg == 0) return LSQR_OK;
   CKL(h, repro_pack(src, n, nseg, stride, h->rbuf, 0, h->s), "repro_pack");
   CKR(allreduce(h, h->rbuf, 2 * n * nseg));
   CKL(h, repro_pack(src, n, nseg, stride, h->rbuf, 1, h->s), "repro_unpack");
@@ -285,7 +286,7 @@ int enqueue_repro(lsqr_t h, int init) {
 int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   SysView& S = h->S;
   cudaStream_t s = h->s;
-  const bool multi = h->nranks > 1;
+  const bool multi = h->multi;
   const bool fused = h->params.fused != 0;
   if (h->repro) {  // NEXT-4: 7 launches (+ 4 x pack/unpack when P > 1), all in lsqr_repro.cu
     if (ev) cudaEventRecord(ev[0], s);
@@ -351,8 +352,8 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
 }
 
 int kernels_per_iteration(lsqr_t h) {
-  if (h->repro) return h->nranks > 1 ? 15 : 7;
-  return h->nranks > 1 ? 9 : (h->params.fused ? 4 : 6);
+  if (h->repro) return h->multi ? 15 : 7;
+  return h->multi ? 9 : (h->params.fused ? 4 : 6);
 }
 
 int build_graph(lsqr_t h) {
@@ -361,7 +362,7 @@ int build_graph(lsqr_t h) {
     h->gexec = nullptr;
   }
   h->graph_ok = false;
-  if (h->nranks > 1 && h->comm_kind == LSQR_COMM_CALLBACK) return LSQR_OK;  // host callback: no capture
+  if (h->multi && h->comm_kind == LSQR_COMM_CALLBACK) return LSQR_OK;  // host callback: no capture
   cudaGraph_t g = nullptr;
   CKC(h, cudaStreamBeginCapture(h->s, cudaStreamCaptureModeThreadLocal));
   int rc = enqueue_iteration(h, nullptr);
@@ -481,8 +482,9 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
     return LSQR_EINVAL;
   if (env->nranks < 1 || env->rank < 0 || env->rank >= env->nranks) return LSQR_EINVAL;
   if ((env->alloc == nullptr) != (env->free == nullptr)) return LSQR_EINVAL;
-  if (env->nranks > 1) {
-    if (env->comm_kind == LSQR_COMM_NCCL && !env->nccl_id) return LSQR_EINVAL;
+  if (env->force_collectives != 0 && env->force_collectives != 1) return LSQR_EINVAL;
+  if (env->nranks > 1 || env->force_collectives) {
+    if (env->comm_kind == LSQR_COMM_NCCL && !env->nccl_id && env->nranks > 1) return LSQR_EINVAL;
     if (env->comm_kind == LSQR_COMM_CALLBACK && !env->allreduce) return LSQR_EINVAL;
     if (env->comm_kind != LSQR_COMM_NCCL && env->comm_kind != LSQR_COMM_CALLBACK) return LSQR_EINVAL;
   }
@@ -517,6 +519,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   h->n_stars = n_stars; h->n_obs = n_obs; h->n_att = n_att; h->n_instr = n_instr; h->n_glob = n_glob;
   h->n_axis = n_axis; h->A0g = A0g; h->I0g = I0g; h->G0g = G0g; h->n_cols_g = n_cols_g;
   h->rank = env->rank; h->nranks = env->nranks; h->device = env->device; h->comm_kind = env->comm_kind;
+  h->multi = env->nranks > 1 || env->force_collectives == 1;
   h->alloc = env->alloc; h->free = env->free; h->alloc_user = env->alloc_user;
   h->cb_allreduce = env->allreduce; h->cb_user = env->allreduce_user;
   h->user_stream = (cudaStream_t)(uintptr_t)env->stream;
@@ -742,10 +745,11 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   if (cudaStreamSynchronize(h->s) != cudaSuccess) return bail(LSQR_ECUDA);
 
   // ---- communicator
-  if (h->nranks > 1 && h->comm_kind == LSQR_COMM_NCCL) {
+  if (h->multi && h->comm_kind == LSQR_COMM_NCCL) {
     if (!nccl_load()) return bail(LSQR_ENCCL);
     ncclUniqueId id;
-    memcpy(id.internal, env->nccl_id, 128);
+    if (env->nccl_id) memcpy(id.internal, env->nccl_id, 128);
+    else if (g_nccl.GetUniqueId(&id) != ncclSuccess) return bail(LSQR_ENCCL);  // 1-rank test communicator
     if (g_nccl.CommInitRank(&h->nccl, h->nranks, id, h->rank) != ncclSuccess) return bail(LSQR_ENCCL);
   }
   *out = h;
@@ -922,7 +926,7 @@ int lsqr_set_reproducible(lsqr_t h, int32_t on) {
     const int64_t L = repro_digits_per_value();
     CKR(dalloc(h, &h->rzd, L * h->n_loc_cols));
     CKR(dalloc(h, &h->rsd, repro_sd_size(h->n_constr)));
-    if (h->nranks > 1) CKR(dalloc(h, &h->rbuf, 2 * std::max<int64_t>(L * h->n_sh, repro_sd_size(h->n_constr))));
+    if (h->multi) CKR(dalloc(h, &h->rbuf, 2 * std::max<int64_t>(L * h->n_sh, repro_sd_size(h->n_constr))));
     CKC(h, cudaMemset(h->rzd, 0, sizeof(long long) * L * h->n_loc_cols));
     CKC(h, cudaMemset(h->rsd, 0, sizeof(long long) * repro_sd_size(h->n_constr)));
   }
@@ -939,7 +943,7 @@ int lsqr_aprod1(lsqr_t h, const double* x_dev, double* y_dev) {
   enter(h);
   CKL(h, launch_aprod1(AP1_PLAIN, S, h->grid, x_dev, y_dev, h->part_rows, h->cpart, h->st, h->s), "aprod1");
   if (h->n_constr > 0) {
-    if (h->nranks == 1) {
+    if (!h->multi) {
       CKL(h, launch_cdot_add(S, h->cpart, nullptr, y_dev + h->n_loc_rows, h->s), "cdot");
     } else {
       CKL(h, launch_beta(3, S, nullptr, 0, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, h->s), "cdot1");
@@ -973,7 +977,7 @@ int lsqr_init(lsqr_t h, const lsqr_solve_params* p) {
   h->params = *p;
   if (h->params.poll_every <= 0) h->params.poll_every = 16;
   SysView& S = h->S;
-  const bool multi = h->nranks > 1;
+  const bool multi = h->multi;
   enter(h);
   DevState st0;
   memset(&st0, 0, sizeof st0);
@@ -1223,7 +1227,7 @@ int lsqr_solve(lsqr_t h, const lsqr_solve_params* p, lsqr_result* res, double* x
   if (res) {
     res->t_iter_mean_s = res->itn > 0 ? ms * 1e-3 / res->itn : 0.0;
     res->t_iter_max_over_ranks_s = res->t_iter_mean_s;
-    if (h->nranks > 1 && h->comm_kind == LSQR_COMM_NCCL) {
+    if (h->multi && h->comm_kind == LSQR_COMM_NCCL) {
       double t = res->t_iter_mean_s;
       CKC(h, cudaMemcpy(h->tmax, &t, sizeof t, cudaMemcpyHostToDevice));
       ncclResult_t r = g_nccl.AllReduce(h->tmax, h->tmax, 1, ncclFloat64, ncclMax, h->nccl, h->s);

@@ -236,3 +236,46 @@ def test_gpu_repro_bitwise_across_rank_counts(cuda_device, P):
         assert same(D[:A0l], D1[5 * sb:5 * se]) and same(D[A0l:], D1[A0:])
         assert same(x[:A0l], ref["x"][5 * sb:5 * se]) and same(x[A0l:], ref["x"][A0:])
         assert same(sev[:A0l], ref["se"][5 * sb:5 * se]) and same(sev[A0l:], ref["se"][A0:])
+
+
+# ------------------------------------------------------------------------------------------------ GPU, NCCL path
+@pytest.mark.gpu
+@pytest.mark.parametrize("mode", ["twopass", "fused", "repro"])
+def test_gpu_nccl_path_forced_on_one_rank(cuda_device, mode):
+    """The multi-rank algorithm (AR1/AR2, or the repro digit reductions) through a REAL NCCL communicator: with
+    lsqr_env.force_collectives a single process builds a 1-rank NCCL communicator (dlopen'ed libnccl, internally
+    generated unique id) and runs every collective of the P > 1 path, captured in the CUDA graph.  NCCL cannot put
+    two ranks on one GPU, so this is how the NCCL plumbing is exercised in a one-GPU run; the results must equal the
+    single-rank path (bit-identical in the reproducible mode)."""
+    import torch
+    import paper_conf_sc_malenzacsbvba24_b200 as avu
+    w = W.C1C.replace(jitter_pct=50)
+    itn = 160 if mode != "repro" else 40
+    kw = dict(itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=True, fused=(mode == "fused"))
+    outs, Ds, prods = [], [], []
+    for force in (False, True):
+        s = avu.Solver.synthetic(w, force_collectives=force)
+        if mode == "repro":
+            s.set_reproducible(True)
+        s.precondition()
+        Ds.append(s.get_precond())
+        xg = torch.ones(s.n_local_cols, dtype=torch.float64, device="cuda")
+        yg = torch.zeros(s.n_local_rows + s.n_constr, dtype=torch.float64, device="cuda")
+        s.aprod1(xg, yg)
+        x2 = torch.zeros_like(xg)
+        s.aprod2(torch.ones_like(yg), x2)
+        prods.append((yg.cpu().numpy(), x2.cpu().numpy()))
+        outs.append(s.solve(**kw))
+        s.close()
+    a, b = outs
+    assert a["itn"] == b["itn"] == itn
+    if mode == "repro":
+        same = lambda p, q: np.array_equal(np.asarray(p).view(np.uint64), np.asarray(q).view(np.uint64))
+        assert same(Ds[0], Ds[1]) and same(a["x"], b["x"]) and same(a["se"], b["se"])
+        assert a["r1norm"] == b["r1norm"] and a["acond"] == b["acond"]
+    else:
+        rel = lambda p, q: np.linalg.norm(p - q) / np.linalg.norm(q)
+        assert np.allclose(Ds[0], Ds[1], rtol=1e-14, atol=0)
+        assert rel(b["x"], a["x"]) <= 1e-9 and abs(b["r1norm"] - a["r1norm"]) <= 1e-10 * a["r1norm"]
+    assert np.allclose(prods[0][0], prods[1][0], rtol=1e-12, atol=1e-12)
+    assert np.allclose(prods[0][1], prods[1][1], rtol=1e-12, atol=1e-12)
