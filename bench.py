@@ -199,7 +199,7 @@ def run_reference(args):
                              "sample": f"full {w.name} system, {len(per)} LSQR iterations after {args.warmup} "
                                        f"warm-up (setup {setup:.1f} s excluded)", "cpu_model": _cpu_model()},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line), flush=True)
+    emit(line)
     return 0
 
 
@@ -360,14 +360,35 @@ def run_ours(args):
     if rank == 0 and n == 1 and args.cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(base, iters=args.cpu_iters, repro=args.repro)
     if rank == 0:
-        print(json.dumps(line), flush=True)
+        emit(line)
     if multi:
         dist.barrier()
         dist.destroy_process_group()
     return 0
 
 
+_JSON_OUT = None
+
+
+def _guard_stdout():
+    """stdout carries exactly one JSON line (rank 0): libraries that print to the C-level stdout (e.g. NCCL's
+    'NCCL version ...' banner at communicator init, on every rank) are redirected to stderr by pointing fd 1 at
+    fd 2; the JSON line goes to a saved duplicate of the original stdout."""
+    global _JSON_OUT
+    if _JSON_OUT is None:
+        sys.stdout.flush()
+        _JSON_OUT = os.fdopen(os.dup(1), "w")
+        os.dup2(2, 1)
+
+
+def emit(line: dict):
+    out = _JSON_OUT if _JSON_OUT is not None else sys.stdout
+    out.write(json.dumps(line) + "\n")
+    out.flush()
+
+
 def main():
+    _guard_stdout()
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=100)
