@@ -15,7 +15,7 @@ namespace lsqr {
 namespace {
 
 constexpr int kL = 5;  // digits
-__device__ __constant__ int kB[kL] = {-8, -48, -88, -128, -168};
+// digit q covers bits [B_q, B_q + 40), B = -8, -48, -88, -128, -168 (docs/REPRO.md)
 
 struct Eda {
   long long d[kL];
