@@ -135,7 +135,10 @@ class Solver:
                     return None
 
             def _free(ptr, user):
-                torch.cuda.caching_allocator_delete(ptr)
+                try:  # (may run from __del__ at interpreter exit, after torch is torn down)
+                    torch.cuda.caching_allocator_delete(ptr)
+                except Exception:
+                    pass
 
             fa, ff = _capi.ALLOC_FN(_alloc), _capi.FREE_FN(_free)
             self._keep += [fa, ff]
