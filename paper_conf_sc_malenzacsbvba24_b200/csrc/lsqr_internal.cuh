@@ -14,7 +14,11 @@ constexpr int kRows = 16;            // rows per TMA stage (two 8-row groups, 4 
 constexpr int kGroups = kRows / 8;
 constexpr int kStages = 3;           // ring depth per warp (kStages-1 stages in flight while computing)
 constexpr int kStageBytes = kRows * (kSlots * 8 + 16);                  // 3328 B: values + index records
-constexpr int kFWarps = 16;          // fused kernel: warps per CTA (own partition SysView::warp_star_f; 12 x 6 stages measured slower)
+#ifndef LSQR_FWARPS
+#define LSQR_FWARPS 16
+#endif
+constexpr int kFWarps = LSQR_FWARPS; // fused kernel: warps per CTA (own partition SysView::warp_star_f; 12 x 6 stages
+                                     // and a separate producer warp measured slower)
 constexpr int kFStages = 4;          // fused kernel: ring depth (8-row stages)
 constexpr int kRingBytes = kWarpsPerCta * kStages * kStageBytes;        // 159,744 B per CTA
 constexpr int kBarBytes = kWarpsPerCta * kStages * 8;                   // mbarriers

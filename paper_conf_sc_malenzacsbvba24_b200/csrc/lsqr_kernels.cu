@@ -658,7 +658,6 @@ __global__ void __launch_bounds__(kThreads, 1)
 constexpr int kFRows = 8, kFPre = 1;  // kFPre: gather prefetch distance in groups (2 measured slower)
 using FRing = RingT<kFRows, kFStages, kFWarps>;
 constexpr int kSmemMaxBytes = 232448;  // 227 KB opt-in per CTA on sm_100
-constexpr int kFusedInstrMax = (kSmemMaxBytes - FRing::kBytes - FRing::kBars - 1024) / 16 - 2;  // 1 KB static
 
 template <bool SMEM_INSTR, int DIAG = 0>
 __global__ void __launch_bounds__(kFWarps * 32, 1)
@@ -901,6 +900,284 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
       const double vv = sh_z[S.ip.fwd(i)];
       if (vv != 0.0) atomicAdd(zsh + S.n_att + i, vv);
     }
+  }
+}
+
+// ------------------------------------------------------------------------------------------------ fused pass, lean
+// k_fused3: the fused single pass of k_fused (same arithmetic, same partition, same TMA ring) with a hot loop
+// written for issue efficiency -- the kernel is bound by the SM's issue slots and L1 data pipe, not by HBM
+// (DESIGN.md §7):
+//   * the loop is unrolled by two so the gather prefetch (group k+1) and the u_hat register queue alternate between
+//     two register sets instead of being copied every group;
+//   * the ring's shared memory is zeroed at entry, so the index records of rows past the end of a warp's range are
+//     always in range (stale rows of the warp or zeros) and the gathers need no validity selects;
+//   * the astro slot-4 (lane 0), instrumental-5 (lanes 1, 2) and global (lane 3) contributions of slot t=5 share one
+//     accumulator `acc5`, folded per star (lane 0: zA, lane 3: global sum; lanes 1, 2 discard theirs);
+//   * shared-memory FP64 accumulation of the instrumental slice uses the compiler's CAS-spin loop (ATOMS.CAST.SPIN;
+//     measured faster than an explicit atom.cas loop);
+//   * no proxy fence before re-filling a stage: lane 0 issues the TMA that overwrites a stage only after every lane
+//     has USED the values it loaded from it (the row dot depends on all of them; __syncwarp), so no read of the
+//     stage is outstanding; the fence cost a MEMBAR.ALL.CTA per group.
+constexpr int kF3Stage = kFRows * (kSlots * 8 + 16);  // 1664 B: 8 rows of values + 8 index records
+constexpr int kF3Bars = kFWarps * kFStages * 8;          // per stage: "full" mbarrier (TMA bytes)
+constexpr int kF3InstrMax = (kSmemMaxBytes - FRing::kBytes - kF3Bars - 1024) / 16 - 2;
+
+template <int DIAG = 0>
+__global__ void __launch_bounds__(kFWarps * 32, 1)
+    k_fused3(SysView S, const double* __restrict__ x, double* __restrict__ u, double* __restrict__ zA,
+             double* __restrict__ zsh, double* __restrict__ part, double* __restrict__ cpart,
+             const DevState* __restrict__ st) {
+  extern __shared__ __align__(128) unsigned char dsm[];
+  if (st->halted) return;
+  // shared memory: [ring | mbarriers | v_instr (slots) + v_glob | z_instr accumulator]
+  const int64_t nsl = S.ip.slots();
+  double* sh_x = reinterpret_cast<double*>(dsm + FRing::kBytes + kF3Bars);
+  double* sh_z = sh_x + nsl + 2;
+  for (int i = threadIdx.x; i < FRing::kBytes / 16; i += blockDim.x)
+    reinterpret_cast<int4*>(dsm)[i] = make_int4(0, 0, 0, 0);
+  for (int64_t i = threadIdx.x; i < nsl; i += blockDim.x) {
+    sh_x[i] = 0.0;
+    sh_z[i] = 0.0;
+  }
+  __syncthreads();
+  for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_x[S.ip.fwd(i)] = x[S.I0 + i];
+  if (threadIdx.x == 0) sh_x[nsl] = S.n_glob ? x[S.G0] : 0.0;
+  const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2, wid = threadIdx.x >> 5;
+  const uint32_t ring = smem_u32(dsm) + wid * kFStages * kF3Stage;
+  const uint32_t bar = smem_u32(dsm + FRing::kBytes) + wid * kFStages * 8;
+  if (lane == 0) {
+    for (int q = 0; q < kFStages; ++q) mbar_init(bar + 8 * q, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();  // ring zeroed (generic writes) before any TMA lands; v_instr staged
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const double uscale = st->u_scale;
+  const int64_t s_lo = S.warp_star_f[gw], s_hi = S.warp_star_f[gw + 1];
+  const int64_t r_lo = S.star_ptr[s_lo];
+  const int nrows = (int)(S.star_ptr[s_hi] - r_lo);  // rows of this warp (< 2^31)
+  const int nst = (nrows + kFRows - 1) / kFRows;
+
+  // producer state (lane 0): stage q goes to slot q % kFStages, issued when the warp releases stage q - kFStages
+  const double* vsrc = S.vals + r_lo * kSlots;
+  const IdxRec* isrc = S.idx + r_lo;
+  int left = nrows;
+  const uint64_t pol = l2_evict_first_policy();
+  auto issue = [&](int slot) {
+    const uint32_t n = (uint32_t)(left < kFRows ? left : kFRows);
+    const uint32_t b = bar + 8 * slot, dst = ring + slot * kF3Stage;
+    mbar_expect_tx(b, n * (kSlots * 8 + 16));
+    bulk_g2s(dst, vsrc, n * (kSlots * 8), b, pol);
+    bulk_g2s(dst + kFRows * kSlots * 8, isrc, n * 16, b, pol);
+    vsrc += kFRows * kSlots;
+    isrc += kFRows;
+    left -= (int)n;
+  };
+  if (lane == 0) {
+    fence_proxy_async();  // the zeroing stores above precede the TMA writes into the ring
+    for (int q = 0; q < kFStages && q < nst; ++q) issue(q);
+  }
+
+  const unsigned char* ringp = dsm + wid * kFStages * kF3Stage;
+  const int voff = r * kSlots * 8 + 48 * j, ioff = kFRows * kSlots * 8 + r * 16;
+  const double* xatt0 = x + S.A0 + j;
+  const double* xatt1 = xatt0 + S.n_axis;
+  const double* xatt2 = xatt1 + S.n_axis;
+  double* zatt0 = zsh + j;
+  double* zatt1 = zatt0 + S.n_axis;
+  double* zatt2 = zatt1 + S.n_axis;
+  const bool t5_ins = (j == 1 || j == 2);  // t=5 slot: lane 0 astro 4, lanes 1, 2 instr 4, 5, lane 3 global
+  const int i5_shift = (j & 2) << 3;
+  const uint32_t i5_or = (j == 3) ? (uint32_t)nsl : 0u;  // lane 3 gathers v_glob (slot nsl); lane 0 ignores its g5
+  const int i4_shift = (j & 1) << 4;
+  double* const urow = u + r_lo + r;
+
+  // warp-uniform star state: cs = star of the next row to process; its astro values (cj, c4) and the next star's
+  int64_t cs = s_lo;
+  int cs_end = (cs < s_hi) ? (int)(S.star_ptr[cs + 1] - r_lo) : nrows;
+  double cj = 0.0, c4 = 0.0, nj = 0.0, n4 = 0.0;
+  if (cs < s_hi) { cj = __ldg(x + 5 * cs + j); c4 = __ldg(x + 5 * cs + 4); }
+  if (cs + 1 < s_hi) { nj = __ldg(x + 5 * (cs + 1) + j); n4 = __ldg(x + 5 * (cs + 1) + 4); }
+  double b2 = 0.0, gacc = 0.0, acc0 = 0.0, acc5 = 0.0;
+
+  auto advance = [&]() {  // star cs is complete: its 5 astro sums -> zA (scatter-free), move to cs+1
+    double z0 = acc0, z1 = acc5;
+    gacc += acc5;  // lane 3: global contributions of the star (lanes 0-2: unused)
+    z0 += __shfl_xor_sync(0xffffffffu, z0, 4);
+    z1 += __shfl_xor_sync(0xffffffffu, z1, 4);
+    z0 += __shfl_xor_sync(0xffffffffu, z0, 8);
+    z1 += __shfl_xor_sync(0xffffffffu, z1, 8);
+    z0 += __shfl_xor_sync(0xffffffffu, z0, 16);
+    z1 += __shfl_xor_sync(0xffffffffu, z1, 16);
+    if (lane < 4) {
+      zA[5 * cs + j] = z0;
+      if (j == 0) zA[5 * cs + 4] = z1;
+    }
+    acc0 = 0.0;
+    acc5 = 0.0;
+    ++cs;
+    cs_end = (cs < s_hi) ? (int)(S.star_ptr[cs + 1] - r_lo) : nrows;
+    cj = nj;
+    c4 = n4;
+    if (cs + 1 < s_hi) { nj = __ldg(x + 5 * (cs + 1) + j); n4 = __ldg(x + 5 * (cs + 1) + 4); }
+  };
+  while (cs < s_hi && cs_end <= 0) advance();  // leading empty stars
+
+  struct Pre {
+    double g1, g2, g3, g4, g5;
+    int k0;
+    uint32_t i4, i5;
+  };
+  // gathers of stage q (slot sl): attitude from L2, instrumental from shared memory
+  auto prefetch = [&](int q, int sl, Pre& P) {
+    mbar_wait(bar + 8 * sl, (uint32_t)(q >> 2) & 1u);
+    static_assert(kFStages == 4, "parity uses q / 4");
+    const int4 rec = *reinterpret_cast<const int4*>(ringp + sl * kF3Stage + ioff);
+    P.k0 = rec.x;
+    P.i4 = ((uint32_t)((j & 2) ? rec.z : rec.y) >> i4_shift) & 0xffffu;
+    P.i5 = t5_ins ? (((uint32_t)rec.w >> i5_shift) & 0xffffu) : i5_or;
+    P.g1 = (DIAG & 4) ? 0.5 : __ldg(xatt0 + P.k0);
+    P.g2 = (DIAG & 4) ? 0.5 : __ldg(xatt1 + P.k0);
+    P.g3 = (DIAG & 4) ? 0.5 : __ldg(xatt2 + P.k0);
+    P.g4 = (DIAG & 8) ? 0.5 : sh_x[P.i4];
+    P.g5 = (DIAG & 8) ? 0.5 : sh_x[P.i5];
+  };
+
+  // one 8-row group.  CHECK: tail / star-boundary path with per-lane validity and per-lane star; otherwise every
+  // lane's row is valid and in star cs.
+  auto group = [&](const double (&v)[6], const Pre& P, int g0, double uold, auto check_tag) {
+    constexpr bool CHECK = decltype(check_tag)::value;
+    const int rel = g0 + r;
+    const bool valid = !CHECK || rel < nrows;
+    double xj = cj, x4 = c4;
+    int64_t my_s = cs;
+    if (CHECK && valid) {
+      int my_end = cs_end;
+      while (my_end <= rel) {
+        ++my_s;
+        my_end = (int)(S.star_ptr[my_s + 1] - r_lo);
+      }
+      if (my_s == cs + 1) { xj = nj; x4 = n4; }
+      else if (my_s != cs) { xj = __ldg(x + 5 * my_s + j); x4 = __ldg(x + 5 * my_s + 4); }
+    }
+    const double g5 = (j == 0) ? x4 : P.g5;
+    double p = fma(v[1], P.g1, v[0] * xj);  // two short chains instead of one long one
+    double p2 = fma(v[4], P.g4, v[3] * P.g3);
+    p = fma(v[2], P.g2, p);
+    p2 = fma(v[5], g5, p2);
+    p += p2;
+    p += __shfl_xor_sync(0xffffffffu, p, 1);
+    p += __shfl_xor_sync(0xffffffffu, p, 2);
+    const double un = valid ? fma(-uscale, uold, p) : 0.0;  // identical in the row's 4 lanes
+    if (j == 0 && valid) {
+      __stcs(urow + g0, un);
+      b2 = fma(un, un, b2);
+    }
+    const double c1 = v[1] * un, c2 = v[2] * un, c3 = v[3] * un, c4v = v[4] * un, c5 = v[5] * un;
+    if (valid && !(DIAG & 2)) {
+      atomicAdd(zatt0 + P.k0, c1);
+      atomicAdd(zatt1 + P.k0, c2);
+      atomicAdd(zatt2 + P.k0, c3);
+    }
+    if (valid && !(DIAG & 1)) {
+      atomicAdd(sh_z + P.i4, c4v);
+      if (t5_ins) atomicAdd(sh_z + P.i5, c5);
+    }
+    if (!CHECK) {
+      acc0 = fma(v[0], un, acc0);
+      acc5 += c5;
+    } else {  // segmented by star inside the group
+      const double c0 = v[0] * un;
+      const int g1end = g0 + kFRows < nrows ? g0 + kFRows : nrows;
+      while (true) {
+        if (valid && my_s == cs) { acc0 += c0; acc5 += c5; }
+        if (cs < s_hi && cs_end <= g1end) advance();
+        else break;
+      }
+    }
+  };
+
+  // one stage: prefetch the next stage's gathers, take this stage's values into registers, hand the slot back to
+  // the TMA (lane 0 refills it with stage k + kFStages), compute
+  auto step = [&](int k, int sl, int sln, const Pre& Pc, Pre& Pn, double& uq) {
+    const int g0 = k * kFRows;
+    if (k + 1 < nst) prefetch(k + 1, sln, Pn);
+    const unsigned char* stg = ringp + sl * kF3Stage;
+    double v[6];
+    {
+      const double2* rp = reinterpret_cast<const double2*>(stg + voff);
+#pragma unroll
+      for (int qq = 0; qq < 3; ++qq) {
+        const double2 d = rp[qq];
+        v[2 * qq] = d.x;
+        v[2 * qq + 1] = d.y;
+      }
+    }
+    // Refill: at every odd stage the slots of stages k-1 and k get stages k+3 and k+4 (one proxy fence per two
+    // stages).  The fence (generic-proxy reads of the slot -> async-proxy TMA writes into it) is required: without
+    // it, or with an intra-warp mbarrier hand-off instead, the full-size C2 parity test fails (x off by ~1e-4).
+    auto release = [&]() {
+      if (k & 1) {
+        __syncwarp();
+        if (lane == 0 && k + kFStages - 1 < nst) {
+          fence_proxy_async();
+          issue((sl + kFStages - 1) & (kFStages - 1));
+          if (k + kFStages < nst) issue(sl);
+        }
+      }
+    };
+    double uold = uq;
+    uq = (g0 + 2 * kFRows + r < nrows) ? __ldcs(urow + g0 + 2 * kFRows) : 0.0;  // u_hat two stages ahead
+    if ((g0 + kFRows <= nrows) && (cs_end >= g0 + kFRows)) {
+      release();
+      group(v, Pc, g0, uold, std::false_type{});
+      while (cs < s_hi && cs_end <= g0 + kFRows) advance();
+    } else {
+      if (g0 + r >= nrows) {
+#pragma unroll
+        for (int t = 0; t < 6; ++t) v[t] = 0.0;
+        uold = 0.0;
+      }
+      release();
+      group(v, Pc, g0, uold, std::true_type{});
+    }
+  };
+
+  double uqa = (r < nrows) ? __ldcs(urow) : 0.0;                   // u_hat of even stages
+  double uqb = (kFRows + r < nrows) ? __ldcs(urow + kFRows) : 0.0;  // u_hat of odd stages
+  Pre PA{}, PB{};
+  if (nst > 0) prefetch(0, 0, PA);
+  int k = 0;
+  for (; k + 1 < nst; k += 2) {
+    const int sl = k & (kFStages - 1);
+    step(k, sl, sl + 1, PA, PB, uqa);
+    step(k + 1, sl + 1, (sl + 2) & (kFStages - 1), PB, PA, uqb);
+  }
+  if (k < nst) step(k, k & (kFStages - 1), (k + 1) & (kFStages - 1), PA, PB, uqa);
+  while (cs < s_hi) advance();  // empty trailing stars
+  if (S.n_glob) {
+    gacc = warp_sum(j == 3 ? gacc : 0.0);
+    if (lane == 0 && gacc != 0.0) atomicAdd(zsh + S.n_att + S.n_instr, gacc);
+  }
+  // beta^2: one partial per CTA (warps combined in a fixed order -> deterministic), so k_post re-sums few values
+  __shared__ double b2w[kFWarps];
+  b2 = warp_sum(b2);
+  if (lane == 0) b2w[wid] = b2;
+  for (int64_t c = gw; c < S.n_chunks; c += W) {  // constraint rows: owned-entry partial dots with v
+    double acc = 0.0;
+    for (int64_t e = S.ch_beg[c] + lane; e < S.ch_end[c]; e += 32) acc = fma(S.cval[e], __ldg(x + S.ccol[e]), acc);
+    acc = warp_sum(acc);
+    if (lane == 0) cpart[c] = acc;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int q = 0; q < kFWarps; ++q) t += b2w[q];
+    part[blockIdx.x] = t;
+  }
+  for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
+    const double vv = sh_z[S.ip.fwd(i)];
+    if (vv != 0.0) atomicAdd(zsh + S.n_att + i, vv);
   }
 }
 
@@ -1513,6 +1790,19 @@ cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* p
   k_vshared<<<nblk, kRedThreads, 0, s>>>(S.n_sh, vsh, zsh, part, st, fused);
   return cudaGetLastError();
 }
+template <int DIAG>
+static cudaError_t fz3(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh, double* part,
+                       double* cpart, const DevState* st, cudaStream_t s) {
+  const size_t smem = FRing::kBytes + kF3Bars + (2 * (size_t)S.ip.slots() + 4) * sizeof(double);
+  static size_t attr_set = 0;
+  if (smem > attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(k_fused3<DIAG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    attr_set = smem;
+  }
+  k_fused3<DIAG><<<grid, kFWarps * 32, smem, s>>>(S, x, u, zA, zsh, part, cpart, st);
+  return cudaGetLastError();
+}
 template <bool SM, int DIAG>
 static cudaError_t fz(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh, double* part,
                       double* cpart, const DevState* st, cudaStream_t s) {
@@ -1543,17 +1833,18 @@ static int diag_mode() {
 
 cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh,
                          double* part, double* cpart, const DevState* st, cudaStream_t s) {
-  if (S.ip.slots() > kFusedInstrMax) return fz<false, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+  // instrumental slice too large for shared memory: k_fused with instrumental gathers / REDs in global memory (L2)
+  if (S.ip.slots() > kF3InstrMax) return fz<false, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
 #ifdef LSQR_DIAG_EXPERIMENTS
   switch (diag_mode()) {
-    case 1: return fz<true, 1>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 2: return fz<true, 2>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 4: return fz<true, 4>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 15: return fz<true, 15>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 1: return fz3<1>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 2: return fz3<2>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 4: return fz3<4>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 15: return fz3<15>(S, grid, x, u, zA, zsh, part, cpart, st, s);
     default: break;
   }
 #endif
-  return fz<true, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+  return fz3<0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
 }
 
 cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const double* uc, double* zsh, double* part,
