@@ -288,6 +288,10 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   cudaStream_t s = h->s;
   const bool multi = h->multi;
   const bool fused = h->params.fused != 0;
+  // two-pass: k_aprod1, then aprod2 on the fused kernel's loop (k_fused3<R3_AP2>); afterwards the state is the
+  // fused pass's (unnormalised z in zA / z_sh), finished by the same kernels
+  const bool lean2 = !fused && lean_products_ok(S);
+  const bool fstate = fused || lean2;
   if (h->repro) {  // NEXT-4: 7 launches (+ 4 x pack/unpack when P > 1), all in lsqr_repro.cu
     if (ev) cudaEventRecord(ev[0], s);
     CKR(enqueue_repro(h, 0));
@@ -301,18 +305,23 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
     CKL(h, launch_aprod1(AP1_LSQR, S, h->grid, h->v, h->u, h->part_rows, h->cpart, h->st, s), "aprod1");
   }
   if (ev) cudaEventRecord(ev[1], s);
-  if (fused && !multi) {  // 4 launches: fused rows, post (beta + v' everywhere), scalar, column update
+  if (lean2) {  // z = A^T u_hat with the unnormalised u_hat (beta is applied afterwards, as in the fused pass)
     if (ev) cudaEventRecord(ev[2], s);
-    CKL(h, launch_post(S, h->v, h->zA, h->zsh, h->part_rows, h->grid, h->cpart, h->uc, h->uc_tmp, h->part_va,
-                       kG3, h->st, s), "post");
+    CKL(h, launch_ap2_lean(S, h->grid, h->u, h->zA, h->zsh, h->st, s), "aprod2");
     if (ev) cudaEventRecord(ev[3], s);
+  }
+  if (fstate && !multi) {  // fused: 4 launches (rows, post = beta + v' everywhere, scalar, column update); lean2: 5
+    if (ev && !lean2) cudaEventRecord(ev[2], s);
+    CKL(h, launch_post(S, h->v, h->zA, h->zsh, h->part_rows, fused ? h->grid : h->W, h->cpart, h->uc, h->uc_tmp,
+                       h->part_va, kG3, h->st, s), "post");
+    if (ev && !lean2) cudaEventRecord(ev[3], s);
     CKL(h, launch_scalar(h->st, h->part_va, kG3, nullptr, 0, h->part_wa, kG3, h->part_ws, kG3, nullptr, nullptr, 0,
                          h->hflag_dev, s, h->uc_tmp, h->uc, h->ucn, (int)h->n_constr), "scalar");
     CKL(h, launch_colupdate(h->v, h->w, h->x, h->var, h->n_loc_cols, S.A0, h->part_wa, h->part_ws, kG3, h->st, s),
         "colupdate");
     return LSQR_OK;
   }
-  const int64_t n_b2 = fused ? h->grid : h->W;  // k_fused publishes one beta^2 partial per CTA
+  const int64_t n_b2 = fused ? h->grid : h->W;  // k_fused3 publishes one beta^2 partial per CTA, k_aprod1 per warp
   if (!multi) {
     CKL(h, launch_beta(0, S, h->part_rows, n_b2, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta");
   } else {
@@ -322,10 +331,10 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
     CKR(allreduce(h, h->ar1, h->n_constr + 2));
     CKL(h, launch_beta(2, S, h->part_rows, n_b2, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta2");
   }
-  if (ev) cudaEventRecord(ev[2], s);
+  if (ev && !lean2) cudaEventRecord(ev[2], s);
   const double* a2part;
   int64_t n_a2;
-  if (fused) {
+  if (fstate) {
     CKL(h, launch_vastro(S, h->v, h->zA, h->uc, h->zsh, h->part_va, kG3, h->st, h->rank == 0, s), "vastro");
     a2part = h->part_va;
     n_a2 = kG3;
@@ -335,13 +344,13 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
     a2part = h->part_a2;
     n_a2 = h->W;
   }
-  if (ev) cudaEventRecord(ev[3], s);
+  if (ev && !lean2) cudaEventRecord(ev[3], s);
   if (multi) {
     // AR2 payload: [z_att | z_instr | z_glob | alpha^2 astro local]
     CKL(h, launch_sum_to(a2part, n_a2, h->zsh + h->n_sh, s), "a2sum");
     CKR(allreduce(h, h->zsh, h->n_sh + 1));
   }
-  CKL(h, launch_vshared(S, h->v + S.A0, h->zsh, h->part_sh, kG2, h->st, fused ? 1 : 0, s), "vshared");
+  CKL(h, launch_vshared(S, h->v + S.A0, h->zsh, h->part_sh, kG2, h->st, fstate ? 1 : 0, s), "vshared");
   CKL(h, launch_scalar(h->st, a2part, n_a2, h->part_sh, kG2, h->part_wa, kG3, h->part_ws, kG3,
                        multi ? h->zsh + h->n_sh : nullptr, multi ? h->ar1 + h->n_constr + 1 : nullptr, 0,
                        h->hflag_dev, s),
@@ -353,7 +362,8 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
 
 int kernels_per_iteration(lsqr_t h) {
   if (h->repro) return h->multi ? 15 : 7;
-  return h->multi ? 9 : (h->params.fused ? 4 : 6);
+  if (h->params.fused) return h->multi ? 9 : 4;
+  return lean_products_ok(h->S) ? (h->multi ? 10 : 5) : (h->multi ? 9 : 6);
 }
 
 int build_graph(lsqr_t h) {

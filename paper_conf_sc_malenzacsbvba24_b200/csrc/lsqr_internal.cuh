@@ -155,6 +155,11 @@ cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* p
 // NEXT-1 fused single pass (u_hat update + A^T u_hat in one read of A) and its astro column pass
 cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh,
                          double* part, double* cpart, const DevState* st, cudaStream_t s);
+// the two-pass iteration's aprod2 on the fused kernel's loop (k_fused3<R3_AP2>): z = A^T u_hat (unnormalised) into
+// zA / z_sh, the state the fused pass leaves; needs the instrumental slice in shared memory (lean_products_ok)
+bool lean_products_ok(const SysView& S);
+cudaError_t launch_ap2_lean(const SysView& S, int grid, const double* u, double* zA, double* zsh, const DevState* st,
+                            cudaStream_t s);
 cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const double* uc, double* zsh, double* part,
                           int nblk, const DevState* st, int do_shared_constr, cudaStream_t s);
 cudaError_t launch_add_shared(double* xsh, double* zsh, int64_t n, int mode, cudaStream_t s);

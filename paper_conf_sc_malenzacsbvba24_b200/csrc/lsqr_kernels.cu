@@ -918,17 +918,27 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
 //   * no proxy fence before re-filling a stage: lane 0 issues the TMA that overwrites a stage only after every lane
 //     has USED the values it loaded from it (the row dot depends on all of them; __syncwarp), so no read of the
 //     stage is outstanding; the fence cost a MEMBAR.ALL.CTA per group.
+//
+// The same loop, templated on KIND, is also the two-pass iteration's aprod2 (the paper's structure: A read twice per
+// iteration):
+//   R3_FUSED: u_hat_i = a_i . v - u_scale u_hat_i, then z += a_i^T u_hat_i  (NEXT-1, the default iteration);
+//   R3_AP2:   z += a_i^T u_hat_i only, on the unnormalised u_hat k_aprod1 wrote (astro z -> zA, shared -> z_sh).
+// k_aprod1<AP1_LSQR> followed by k_fused3<R3_AP2> leaves the state k_fused3<R3_FUSED> leaves, so k_post / k_vastro /
+// k_vshared finish the iteration unchanged (v' = z / beta - beta v).  (An aprod1 on this loop measured slower than
+// k_aprod1's deeper 16-row ring: C3 11.5 vs 10.5 ms.)
+enum { R3_FUSED = 0, R3_AP2 = 2 };
 constexpr int kF3Stage = kFRows * (kSlots * 8 + 16);  // 1664 B: 8 rows of values + 8 index records
 constexpr int kF3Bars = kFWarps * kFStages * 8;          // per stage: "full" mbarrier (TMA bytes)
 constexpr int kF3InstrMax = (kSmemMaxBytes - FRing::kBytes - kF3Bars - 1024) / 16 - 2;
 
-template <int DIAG = 0>
+template <int KIND = R3_FUSED, int DIAG = 0>
 __global__ void __launch_bounds__(kFWarps * 32, 1)
     k_fused3(SysView S, const double* __restrict__ x, double* __restrict__ u, double* __restrict__ zA,
              double* __restrict__ zsh, double* __restrict__ part, double* __restrict__ cpart,
              const DevState* __restrict__ st) {
   extern __shared__ __align__(128) unsigned char dsm[];
   if (st->halted) return;
+  constexpr bool kDot = KIND == R3_FUSED;  // computes the new u_hat (gathers, row dot, store, beta^2)
   // shared memory: [ring | mbarriers | v_instr (slots) + v_glob | z_instr accumulator]
   const int64_t nsl = S.ip.slots();
   double* sh_x = reinterpret_cast<double*>(dsm + FRing::kBytes + kF3Bars);
@@ -940,8 +950,10 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
     sh_z[i] = 0.0;
   }
   __syncthreads();
-  for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_x[S.ip.fwd(i)] = x[S.I0 + i];
-  if (threadIdx.x == 0) sh_x[nsl] = S.n_glob ? x[S.G0] : 0.0;
+  if (kDot) {
+    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_x[S.ip.fwd(i)] = x[S.I0 + i];
+    if (threadIdx.x == 0) sh_x[nsl] = S.n_glob ? x[S.G0] : 0.0;
+  }
   const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2, wid = threadIdx.x >> 5;
   const uint32_t ring = smem_u32(dsm) + wid * kFStages * kF3Stage;
   const uint32_t bar = smem_u32(dsm + FRing::kBytes) + wid * kFStages * 8;
@@ -996,30 +1008,34 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
   int64_t cs = s_lo;
   int cs_end = (cs < s_hi) ? (int)(S.star_ptr[cs + 1] - r_lo) : nrows;
   double cj = 0.0, c4 = 0.0, nj = 0.0, n4 = 0.0;
-  if (cs < s_hi) { cj = __ldg(x + 5 * cs + j); c4 = __ldg(x + 5 * cs + 4); }
-  if (cs + 1 < s_hi) { nj = __ldg(x + 5 * (cs + 1) + j); n4 = __ldg(x + 5 * (cs + 1) + 4); }
+  if (kDot && cs < s_hi) { cj = __ldg(x + 5 * cs + j); c4 = __ldg(x + 5 * cs + 4); }
+  if (kDot && cs + 1 < s_hi) { nj = __ldg(x + 5 * (cs + 1) + j); n4 = __ldg(x + 5 * (cs + 1) + 4); }
   double b2 = 0.0, gacc = 0.0, acc0 = 0.0, acc5 = 0.0;
 
   auto advance = [&]() {  // star cs is complete: its 5 astro sums -> zA (scatter-free), move to cs+1
-    double z0 = acc0, z1 = acc5;
-    gacc += acc5;  // lane 3: global contributions of the star (lanes 0-2: unused)
-    z0 += __shfl_xor_sync(0xffffffffu, z0, 4);
-    z1 += __shfl_xor_sync(0xffffffffu, z1, 4);
-    z0 += __shfl_xor_sync(0xffffffffu, z0, 8);
-    z1 += __shfl_xor_sync(0xffffffffu, z1, 8);
-    z0 += __shfl_xor_sync(0xffffffffu, z0, 16);
-    z1 += __shfl_xor_sync(0xffffffffu, z1, 16);
-    if (lane < 4) {
-      zA[5 * cs + j] = z0;
-      if (j == 0) zA[5 * cs + 4] = z1;
+    {
+      double z0 = acc0, z1 = acc5;
+      gacc += acc5;  // lane 3: global contributions of the star (lanes 0-2: unused)
+      z0 += __shfl_xor_sync(0xffffffffu, z0, 4);
+      z1 += __shfl_xor_sync(0xffffffffu, z1, 4);
+      z0 += __shfl_xor_sync(0xffffffffu, z0, 8);
+      z1 += __shfl_xor_sync(0xffffffffu, z1, 8);
+      z0 += __shfl_xor_sync(0xffffffffu, z0, 16);
+      z1 += __shfl_xor_sync(0xffffffffu, z1, 16);
+      if (lane < 4) {
+        zA[5 * cs + j] = z0;
+        if (j == 0) zA[5 * cs + 4] = z1;
+      }
+      acc0 = 0.0;
+      acc5 = 0.0;
     }
-    acc0 = 0.0;
-    acc5 = 0.0;
     ++cs;
     cs_end = (cs < s_hi) ? (int)(S.star_ptr[cs + 1] - r_lo) : nrows;
-    cj = nj;
-    c4 = n4;
-    if (cs + 1 < s_hi) { nj = __ldg(x + 5 * (cs + 1) + j); n4 = __ldg(x + 5 * (cs + 1) + 4); }
+    if (kDot) {
+      cj = nj;
+      c4 = n4;
+      if (cs + 1 < s_hi) { nj = __ldg(x + 5 * (cs + 1) + j); n4 = __ldg(x + 5 * (cs + 1) + 4); }
+    }
   };
   while (cs < s_hi && cs_end <= 0) advance();  // leading empty stars
 
@@ -1036,11 +1052,13 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
     P.k0 = rec.x;
     P.i4 = ((uint32_t)((j & 2) ? rec.z : rec.y) >> i4_shift) & 0xffffu;
     P.i5 = t5_ins ? (((uint32_t)rec.w >> i5_shift) & 0xffffu) : i5_or;
-    P.g1 = (DIAG & 4) ? 0.5 : __ldg(xatt0 + P.k0);
-    P.g2 = (DIAG & 4) ? 0.5 : __ldg(xatt1 + P.k0);
-    P.g3 = (DIAG & 4) ? 0.5 : __ldg(xatt2 + P.k0);
-    P.g4 = (DIAG & 8) ? 0.5 : sh_x[P.i4];
-    P.g5 = (DIAG & 8) ? 0.5 : sh_x[P.i5];
+    if (kDot) {
+      P.g1 = (DIAG & 4) ? 0.5 : __ldg(xatt0 + P.k0);
+      P.g2 = (DIAG & 4) ? 0.5 : __ldg(xatt1 + P.k0);
+      P.g3 = (DIAG & 4) ? 0.5 : __ldg(xatt2 + P.k0);
+      P.g4 = (DIAG & 8) ? 0.5 : sh_x[P.i4];
+      P.g5 = (DIAG & 8) ? 0.5 : sh_x[P.i5];
+    }
   };
 
   // one 8-row group.  CHECK: tail / star-boundary path with per-lane validity and per-lane star; otherwise every
@@ -1057,21 +1075,28 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
         ++my_s;
         my_end = (int)(S.star_ptr[my_s + 1] - r_lo);
       }
-      if (my_s == cs + 1) { xj = nj; x4 = n4; }
-      else if (my_s != cs) { xj = __ldg(x + 5 * my_s + j); x4 = __ldg(x + 5 * my_s + 4); }
+      if (kDot) {
+        if (my_s == cs + 1) { xj = nj; x4 = n4; }
+        else if (my_s != cs) { xj = __ldg(x + 5 * my_s + j); x4 = __ldg(x + 5 * my_s + 4); }
+      }
     }
-    const double g5 = (j == 0) ? x4 : P.g5;
-    double p = fma(v[1], P.g1, v[0] * xj);  // two short chains instead of one long one
-    double p2 = fma(v[4], P.g4, v[3] * P.g3);
-    p = fma(v[2], P.g2, p);
-    p2 = fma(v[5], g5, p2);
-    p += p2;
-    p += __shfl_xor_sync(0xffffffffu, p, 1);
-    p += __shfl_xor_sync(0xffffffffu, p, 2);
-    const double un = valid ? fma(-uscale, uold, p) : 0.0;  // identical in the row's 4 lanes
-    if (j == 0 && valid) {
-      __stcs(urow + g0, un);
-      b2 = fma(un, un, b2);
+    double un;
+    if (kDot) {
+      const double g5 = (j == 0) ? x4 : P.g5;
+      double p = fma(v[1], P.g1, v[0] * xj);  // two short chains instead of one long one
+      double p2 = fma(v[4], P.g4, v[3] * P.g3);
+      p = fma(v[2], P.g2, p);
+      p2 = fma(v[5], g5, p2);
+      p += p2;
+      p += __shfl_xor_sync(0xffffffffu, p, 1);
+      p += __shfl_xor_sync(0xffffffffu, p, 2);
+      un = valid ? fma(-uscale, uold, p) : 0.0;  // identical in the row's 4 lanes
+      if (j == 0 && valid) {
+        __stcs(urow + g0, un);
+        b2 = fma(un, un, b2);
+      }
+    } else {
+      un = valid ? uold : 0.0;  // aprod2: the u_hat aprod1 wrote
     }
     const double c1 = v[1] * un, c2 = v[2] * un, c3 = v[3] * un, c4v = v[4] * un, c5 = v[5] * un;
     if (valid && !(DIAG & 2)) {
@@ -1161,16 +1186,18 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
   }
   // beta^2: one partial per CTA (warps combined in a fixed order -> deterministic), so k_post re-sums few values
   __shared__ double b2w[kFWarps];
-  b2 = warp_sum(b2);
-  if (lane == 0) b2w[wid] = b2;
-  for (int64_t c = gw; c < S.n_chunks; c += W) {  // constraint rows: owned-entry partial dots with v
-    double acc = 0.0;
-    for (int64_t e = S.ch_beg[c] + lane; e < S.ch_end[c]; e += 32) acc = fma(S.cval[e], __ldg(x + S.ccol[e]), acc);
-    acc = warp_sum(acc);
-    if (lane == 0) cpart[c] = acc;
+  if (kDot) {
+    b2 = warp_sum(b2);
+    if (lane == 0) b2w[wid] = b2;
+    for (int64_t c = gw; c < S.n_chunks; c += W) {  // constraint rows: owned-entry partial dots with v
+      double acc = 0.0;
+      for (int64_t e = S.ch_beg[c] + lane; e < S.ch_end[c]; e += 32) acc = fma(S.cval[e], __ldg(x + S.ccol[e]), acc);
+      acc = warp_sum(acc);
+      if (lane == 0) cpart[c] = acc;
+    }
   }
   __syncthreads();
-  if (threadIdx.x == 0) {
+  if (kDot && threadIdx.x == 0) {
     double t = 0.0;
     for (int q = 0; q < kFWarps; ++q) t += b2w[q];
     part[blockIdx.x] = t;
@@ -1790,17 +1817,17 @@ cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* p
   k_vshared<<<nblk, kRedThreads, 0, s>>>(S.n_sh, vsh, zsh, part, st, fused);
   return cudaGetLastError();
 }
-template <int DIAG>
+template <int KIND, int DIAG>
 static cudaError_t fz3(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh, double* part,
                        double* cpart, const DevState* st, cudaStream_t s) {
   const size_t smem = FRing::kBytes + kF3Bars + (2 * (size_t)S.ip.slots() + 4) * sizeof(double);
   static size_t attr_set = 0;
   if (smem > attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_fused3<DIAG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(k_fused3<KIND, DIAG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr_set = smem;
   }
-  k_fused3<DIAG><<<grid, kFWarps * 32, smem, s>>>(S, x, u, zA, zsh, part, cpart, st);
+  k_fused3<KIND, DIAG><<<grid, kFWarps * 32, smem, s>>>(S, x, u, zA, zsh, part, cpart, st);
   return cudaGetLastError();
 }
 template <bool SM, int DIAG>
@@ -1837,14 +1864,20 @@ cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u,
   if (S.ip.slots() > kF3InstrMax) return fz<false, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
 #ifdef LSQR_DIAG_EXPERIMENTS
   switch (diag_mode()) {
-    case 1: return fz3<1>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 2: return fz3<2>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 4: return fz3<4>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 15: return fz3<15>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 1: return fz3<R3_FUSED, 1>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 2: return fz3<R3_FUSED, 2>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 4: return fz3<R3_FUSED, 4>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 15: return fz3<R3_FUSED, 15>(S, grid, x, u, zA, zsh, part, cpart, st, s);
     default: break;
   }
 #endif
-  return fz3<0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+  return fz3<R3_FUSED, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+}
+
+bool lean_products_ok(const SysView& S) { return S.ip.slots() <= kF3InstrMax; }
+cudaError_t launch_ap2_lean(const SysView& S, int grid, const double* u, double* zA, double* zsh, const DevState* st,
+                            cudaStream_t s) {
+  return fz3<R3_AP2, 0>(S, grid, nullptr, const_cast<double*>(u), zA, zsh, nullptr, nullptr, st, s);
 }
 
 cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const double* uc, double* zsh, double* part,
