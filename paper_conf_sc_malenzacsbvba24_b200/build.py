@@ -52,6 +52,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC,-O2",
            "-Xptxas", "-warn-spills", "-I", os.path.join(ROOT, "include"), "-I", CSRC, "-I", _nccl_include(),
            "-o", tmp] + [os.path.join(CSRC, s) for s in SOURCES] + ["-ldl"]
+    extra = os.environ.get("LSQR_NVCC_EXTRA", "").split()  # experiment builds only (e.g. -DLSQR_DIAG_EXPERIMENTS)
+    cmd[1:1] = extra
     if verbose:
         print(" ".join(cmd), file=sys.stderr)
     subprocess.check_call(cmd)
