@@ -172,12 +172,23 @@ def config_block(w, n, args, extra=None):
     return c
 
 
+def workload_of(args):
+    """The named configuration, with the shared-slice dimensions optionally overridden (SURVEY §8(d) sensitivity
+    sweep: n_att and n_instr on the C3 shape)."""
+    w = W.CONFIGS[args.config]
+    if args.n_att:
+        w = w.replace(n_att=args.n_att, name=f"{w.name}-att{args.n_att}")
+    if args.n_instr:
+        w = w.replace(n_instr=args.n_instr, name=f"{w.name}-instr{args.n_instr}")
+    return w
+
+
 # ------------------------------------------------------------------------------------------------ reference arm
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
-    base = W.CONFIGS[args.config]
+    base = workload_of(args)
     w = base
     import oracle
     t0 = time.perf_counter()
@@ -221,7 +232,7 @@ def run_ours(args):
             dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", local))
         else:  # test mode: gloo + the library's host-callback communicator (ranks may share one GPU)
             dist.init_process_group("gloo", rank=rank, world_size=world)
-    base = W.CONFIGS[args.config]
+    base = workload_of(args)
     w = base.per_gpu(n) if n > 1 else base
     w = w.replace(name=base.name)
     def comm_kw():
@@ -302,7 +313,7 @@ def run_ours(args):
         s.set_reproducible(True)
     t0 = time.perf_counter()
     s.precondition()
-    s.init(itn_limit=2 * K + 2 * Wm + 10, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=True,
+    s.init(itn_limit=4 * K + 2 * Wm + 10, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=True,
            fused=args.fused)
     s.sync()
     t_setup = time.perf_counter() - t0
@@ -317,6 +328,12 @@ def run_ours(args):
         barrier()
         r = s.iterate_timed(K)
         barrier()
+        # 3 repetitions of the K-iteration measurement, median and min reported
+        reps = [t_pass1]
+        for _ in range(2):
+            reps.append(s.iterate_events(K))
+            barrier()
+    reps = [max_over_ranks(t) / K for t in reps]
     t_ms = max_over_ranks(t_pass1)
     ap1_ms = max_over_ranks(r["aprod1_ms"] / K)
     ap2_ms = max_over_ranks(r["aprod2_ms"] / K)
@@ -347,6 +364,8 @@ def run_ours(args):
         "ms_per_step": ms_step, "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
         "data": "synthetic",
         "config": config_block(w, n, args, {"setup_s": round(t_setup, 3)}),
+        "repetitions": {"ms_per_step": [round(t, 5) for t in reps], "median": round(statistics.median(reps), 5),
+                        "min": round(min(reps), 5), "note": "value = repetition 1 (the first K-step pass)"},
         "roofline": {"bound": "hbm", "kernel": kname, "achieved": round(achieved, 1), "peak": peak,
                      "peak_kind": f"{peak_kind} (MEASURED_PEAKS.json hbm_gbs, copy; burst)", "unit": "GB/s",
                      "frac": round(achieved / peak, 4), "traffic": load_traffic(w.name if n == 1 else None, kname),
@@ -411,6 +430,8 @@ def main():
     ap.add_argument("--no-e2e", dest="e2e", action="store_false")
     ap.add_argument("--no-cpu-baseline", dest="cpu_baseline", action="store_false")
     ap.add_argument("--cpu-iters", type=int, default=3)
+    ap.add_argument("--n-att", type=int, default=0, help="override n_att (multiple of 3, >= 12; sensitivity sweep)")
+    ap.add_argument("--n-instr", type=int, default=0, help="override n_instr (multiple of 6; sensitivity sweep)")
     ap.add_argument("--fused", dest="fused", action="store_true", default=True,
                     help="fused single-pass iteration (SURVEY 8(f) NEXT-1; default)")
     ap.add_argument("--two-pass", dest="fused", action="store_false", help="two-pass iteration (aprod1 then aprod2)")
