@@ -113,6 +113,7 @@ struct SysView {
   InstrPerm ip;  // IdxRec instrumental fields hold ip.fwd(column); shared-memory arrays have ip.slots() entries
   // shared-column constraint entries grouped by shared column (CSC) over [scs_lo, scs_hi) (rank 0 only)
   int64_t scs_lo, scs_hi; const int64_t* scs_ptr; const int32_t* scs_k; const int64_t* scs_e;
+  int32_t f3_zrep, f3_arep;  // k_fused3 launch only: shared-memory accumulator copies (set by its launcher)
 };
 
 enum { AP1_LSQR = 0, AP1_PLAIN = 1 };

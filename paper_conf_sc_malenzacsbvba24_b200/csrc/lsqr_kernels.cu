@@ -6,6 +6,7 @@
 // t=5 {astro 4, instr 4, instr 5, global}[j].  Each of the 6 loads of a warp instruction reads 8 rows x 32
 // contiguous bytes, so every fetched byte of A is used; the 4 lanes of a row hit 4 consecutive attitude columns,
 // which makes the attitude gathers (aprod1) and REDs (aprod2) sector-coalesced.
+#include <algorithm>
 #include <cstdlib>
 #include <type_traits>
 
@@ -655,257 +656,12 @@ __global__ void __launch_bounds__(kThreads, 1)
 // algebraically the P&S step b (u = u_hat/beta).  Astro z goes to zA (scatter-free, per star), the shared slice to
 // z_sh exactly as in aprod2.  The ring is shallower (8-row stages) because v_instr (gathers) and z_instr
 // (accumulator) both live in shared memory.
-constexpr int kFRows = 8, kFPre = 1;  // kFPre: gather prefetch distance in groups (2 measured slower)
+constexpr int kFRows = 8;
 using FRing = RingT<kFRows, kFStages, kFWarps>;
 constexpr int kSmemMaxBytes = 232448;  // 227 KB opt-in per CTA on sm_100
 
-template <bool SMEM_INSTR, int DIAG = 0>
-__global__ void __launch_bounds__(kFWarps * 32, 1)
-    k_fused(SysView S, const double* __restrict__ x, double* __restrict__ u, double* __restrict__ zA,
-            double* __restrict__ zsh, double* __restrict__ part, double* __restrict__ cpart,
-            const DevState* __restrict__ st) {
-  extern __shared__ __align__(128) unsigned char dsm[];
-  if (st->halted) return;
-  // shared memory: [ring | mbarriers | v_instr (n_instr) + v_glob | z_instr accumulator (n_instr)]
-  const int64_t nsl = S.ip.slots();
-  double* sh_x = reinterpret_cast<double*>(dsm + FRing::kBytes + FRing::kBars);
-  double* sh_z = sh_x + nsl + 2;
-  if (SMEM_INSTR) {
-    for (int64_t i = threadIdx.x; i < nsl; i += blockDim.x) {
-      sh_x[i] = 0.0;
-      sh_z[i] = 0.0;
-    }
-    __syncthreads();
-    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_x[S.ip.fwd(i)] = x[S.I0 + i];
-    if (threadIdx.x == 0) sh_x[nsl] = S.n_glob ? x[S.G0] : 0.0;
-    __syncthreads();
-  }
-  const int lane = threadIdx.x & 31, j = lane & 3, r = lane >> 2, wid = threadIdx.x >> 5;
-  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int64_t W = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const double uscale = st->u_scale;
-  const int64_t s_lo = S.warp_star_f[gw], s_hi = S.warp_star_f[gw + 1];
-  const int64_t r_lo = S.star_ptr[s_lo];
-  const int nrows = (int)(S.star_ptr[s_hi] - r_lo);  // rows of this warp (< 2^31)
-  FRing R;
-  R.setup(S, dsm, wid, lane, r_lo, r_lo + nrows);
-  R.prologue(lane);
-  // per-lane loop invariants
-  const double* xatt0 = x + S.A0 + j;
-  const double* xatt1 = xatt0 + S.n_axis;
-  const double* xatt2 = xatt1 + S.n_axis;
-  double* zatt0 = zsh + j;
-  double* zatt1 = zatt0 + S.n_axis;
-  double* zatt2 = zatt1 + S.n_axis;
-  const double* xins_g = x + S.I0;      // (non-smem fallback)
-  double* zins_g = zsh + S.n_att;
-  const double vglob_g = S.n_glob ? __ldg(x + S.G0) : 0.0;
-  const double m0 = (j == 0) ? 1.0 : 0.0;                 // lane 0 of a row holds astro slot 4 at t=5
-  const double m3 = (j == 3 && S.n_glob) ? 1.0 : 0.0;     // lane 3 holds the global slot at t=5
-  const bool t5_ins = (j == 1 || j == 2);                 // lanes 1, 2 hold instr 4, 5 at t=5
-  double* const urow = u + r_lo + r;
-
-  // warp-uniform star state: cs = star of the next row to process; its astro values (cj, c4) and the next star's
-  int64_t cs = s_lo;
-  int cs_end = (cs < s_hi) ? (int)(S.star_ptr[cs + 1] - r_lo) : nrows;
-  double cj = 0.0, c4 = 0.0, nj = 0.0, n4 = 0.0;
-  if (cs < s_hi) { cj = __ldg(x + 5 * cs + j); c4 = __ldg(x + 5 * cs + 4); }
-  if (cs + 1 < s_hi) { nj = __ldg(x + 5 * (cs + 1) + j); n4 = __ldg(x + 5 * (cs + 1) + 4); }
-  double b2 = 0.0, gacc = 0.0, acc0 = 0.0, acc1 = 0.0;
-
-  auto advance = [&]() {  // star cs is complete: its 5 astro sums -> zA (scatter-free), move to cs+1
-    double z0 = acc0, z1 = acc1;
-    z0 += __shfl_xor_sync(0xffffffffu, z0, 4);
-    z0 += __shfl_xor_sync(0xffffffffu, z0, 8);
-    z0 += __shfl_xor_sync(0xffffffffu, z0, 16);
-    z1 += __shfl_xor_sync(0xffffffffu, z1, 4);
-    z1 += __shfl_xor_sync(0xffffffffu, z1, 8);
-    z1 += __shfl_xor_sync(0xffffffffu, z1, 16);
-    if (lane < 4) {
-      zA[5 * cs + j] = z0;
-      if (j == 0) zA[5 * cs + 4] = z1;
-    }
-    acc0 = 0.0;
-    acc1 = 0.0;
-    ++cs;
-    cs_end = (cs < s_hi) ? (int)(S.star_ptr[cs + 1] - r_lo) : nrows;
-    cj = nj;
-    c4 = n4;
-    if (cs + 1 < s_hi) { nj = __ldg(x + 5 * (cs + 1) + j); n4 = __ldg(x + 5 * (cs + 1) + 4); }
-  };
-  while (cs < s_hi && cs_end <= 0) advance();  // leading empty stars
-
-  // one 8-row group: gathers, row dot, u_hat update, contributions.  CHECK: tail / star-boundary path with
-  // per-lane validity and per-lane star; otherwise every lane's row is valid and in star cs.
-  // gathers of one 8-row group (attitude from L2, instrumental from shared memory), issued one group ahead of
-  // their use so their latency overlaps the previous group's arithmetic and scatters
-  struct Pre {
-    double g1, g2, g3, g4, g5;
-    int k0;
-    uint32_t i4, i5;
-  };
-  auto prefetch = [&](const unsigned char* stg, int g0) {
-    Pre P;
-    const bool valid = g0 + r < nrows;
-    const int4 q = *reinterpret_cast<const int4*>(stg + kFRows * kSlots * 8 + r * 16);
-    IdxRec rec;
-    rec.k0 = valid ? q.x : 0;
-    rec.ic01 = valid ? (uint32_t)q.y : 0u;
-    rec.ic23 = valid ? (uint32_t)q.z : 0u;
-    rec.ic45 = valid ? (uint32_t)q.w : 0u;
-    P.k0 = rec.k0;
-    P.i4 = ic4_of(rec, j);
-    P.i5 = (j == 3) ? (uint32_t)nsl : ic5_of(rec, j);
-    P.g1 = (DIAG & 4) ? 0.5 : __ldg(xatt0 + P.k0);
-    P.g2 = (DIAG & 4) ? 0.5 : __ldg(xatt1 + P.k0);
-    P.g3 = (DIAG & 4) ? 0.5 : __ldg(xatt2 + P.k0);
-    if (SMEM_INSTR) {
-      P.g4 = (DIAG & 8) ? 0.5 : sh_x[P.i4];
-      P.g5 = (DIAG & 8) ? 0.5 : sh_x[P.i5];
-    } else {
-      P.i5 = ic5_of(rec, j);
-      P.g4 = __ldg(xins_g + P.i4);
-      P.g5 = (j == 3) ? vglob_g : __ldg(xins_g + P.i5);
-    }
-    return P;
-  };
-
-  // one 8-row group: row dot, u_hat update, contributions.  CHECK: tail / star-boundary path with per-lane
-  // validity and per-lane star; otherwise every lane's row is valid and in star cs.
-  auto group = [&](const double (&v)[6], const Pre& P, int g0, double uold, auto check_tag) {
-    constexpr bool CHECK = decltype(check_tag)::value;
-    const int rel = g0 + r;
-    const bool valid = !CHECK || rel < nrows;
-    double xj = cj, x4 = c4;
-    int64_t my_s = cs;
-    if (CHECK && valid) {
-      int my_end = cs_end;
-      while (my_end <= rel) {
-        ++my_s;
-        my_end = (int)(S.star_ptr[my_s + 1] - r_lo);
-      }
-      if (my_s == cs + 1) { xj = nj; x4 = n4; }
-      else if (my_s != cs) { xj = __ldg(x + 5 * my_s + j); x4 = __ldg(x + 5 * my_s + 4); }
-    }
-    const double g5 = (j == 0) ? x4 : P.g5;
-    double p = fma(v[1], P.g1, v[0] * xj);  // two short chains instead of one long one
-    double p2 = fma(v[4], P.g4, v[3] * P.g3);
-    p = fma(v[2], P.g2, p);
-    p2 = fma(v[5], g5, p2);
-    p += p2;
-    p += __shfl_xor_sync(0xffffffffu, p, 1);
-    p += __shfl_xor_sync(0xffffffffu, p, 2);
-    const double un = valid ? p - uscale * uold : 0.0;  // identical in the row's 4 lanes
-    if (j == 0 && valid) {
-      __stcs(urow + g0, un);
-      b2 = fma(un, un, b2);
-    }
-    const double c1 = v[1] * un, c2 = v[2] * un, c3 = v[3] * un, c4v = v[4] * un, c5 = v[5] * un;
-    if (valid && !(DIAG & 2)) {
-      atomicAdd(zatt0 + P.k0, c1);
-      atomicAdd(zatt1 + P.k0, c2);
-      atomicAdd(zatt2 + P.k0, c3);
-    }
-    if (SMEM_INSTR) {
-      double* ia[2] = {sh_z + P.i4, sh_z + P.i5};
-      const double iv[2] = {c4v, c5};
-      const bool ion[2] = {valid && !(DIAG & 1), valid && t5_ins && !(DIAG & 1)};
-      smem_add_n<2>(ia, iv, ion);
-    } else if (valid) {
-      atomicAdd(zins_g + P.i4, c4v);
-      if (t5_ins) atomicAdd(zins_g + P.i5, c5);
-    }
-    gacc = fma(c5, m3, gacc);
-    const double c0 = v[0] * un, c5a = c5 * m0;
-    if (!CHECK) {
-      acc0 += c0;
-      acc1 += c5a;
-    } else {  // segmented by star inside the group
-      const int g1end = g0 + 8 < nrows ? g0 + 8 : nrows;
-      while (true) {
-        if (valid && my_s == cs) { acc0 += c0; acc1 += c5a; }
-        if (cs < s_hi && cs_end <= g1end) advance();
-        else break;
-      }
-    }
-  };
-
-  const int nst = (nrows + kFRows - 1) / kFRows;
-  double uq0 = (r < nrows) ? __ldcs(urow) : 0.0;           // u_hat of stage k (register queue, 2 deep;
-  double uq1 = (kFRows + r < nrows) ? __ldcs(urow + kFRows) : 0.0;  // streaming loads: evict-first in L2)
-  // gathers run kFPre groups ahead of their use (the stages they read are held in the ring until consumed)
-  Pre Pc{}, Pn1{};
-  if (nst > 0) Pc = prefetch(R.wait(), 0);
-  if (kFPre > 1 && nst > 1) Pn1 = prefetch(R.wait_ahead(1), kFRows);
-  for (int k = 0; k < nst; ++k) {
-    const int g0 = k * kFRows;
-    const double uold = uq0;
-    uq0 = uq1;
-    uq1 = (g0 + 2 * kFRows + r < nrows) ? __ldcs(urow + g0 + 2 * kFRows) : 0.0;
-    const unsigned char* stg = R.wait();
-    Pre Pn{};
-    if (k + kFPre < nst) Pn = prefetch(R.wait_ahead(kFPre), g0 + kFPre * kFRows);
-    double v[6];
-    {
-      const double2* rp = reinterpret_cast<const double2*>(stg + r * kSlots * 8 + 48 * j);
-#pragma unroll
-      for (int qq = 0; qq < 3; ++qq) {
-        const double2 d = rp[qq];
-        v[2 * qq] = d.x;
-        v[2 * qq + 1] = d.y;
-      }
-      if (g0 + r >= nrows) {
-#pragma unroll
-        for (int t = 0; t < 6; ++t) v[t] = 0.0;
-      }
-    }
-    R.release(lane);  // the stage's data is in registers: refill its slot now
-    const bool fast = (g0 + kFRows <= nrows) && (cs_end >= g0 + kFRows);
-    if (fast) {
-      group(v, Pc, g0, uold, std::false_type{});
-      while (cs < s_hi && cs_end <= g0 + kFRows) advance();
-    } else {
-      group(v, Pc, g0, uold, std::true_type{});
-    }
-    if (kFPre > 1) {
-      Pc = Pn1;
-      Pn1 = Pn;
-    } else {
-      Pc = Pn;
-    }
-  }
-  while (cs < s_hi) advance();  // empty trailing stars
-  if (S.n_glob) {
-    gacc = warp_sum(gacc);
-    if (lane == 0 && gacc != 0.0) atomicAdd(zsh + S.n_att + S.n_instr, gacc);
-  }
-  // beta^2: one partial per CTA (warps combined in a fixed order -> deterministic), so k_post re-sums few values
-  __shared__ double b2w[kFWarps];
-  b2 = warp_sum(b2);
-  if (lane == 0) b2w[wid] = b2;
-  for (int64_t c = gw; c < S.n_chunks; c += W) {  // constraint rows: owned-entry partial dots with v
-    double acc = 0.0;
-    for (int64_t e = S.ch_beg[c] + lane; e < S.ch_end[c]; e += 32) acc = fma(S.cval[e], __ldg(x + S.ccol[e]), acc);
-    acc = warp_sum(acc);
-    if (lane == 0) cpart[c] = acc;
-  }
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    double t = 0.0;
-    for (int q = 0; q < kFWarps; ++q) t += b2w[q];
-    part[blockIdx.x] = t;
-  }
-  if (SMEM_INSTR) {
-    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
-      const double vv = sh_z[S.ip.fwd(i)];
-      if (vv != 0.0) atomicAdd(zsh + S.n_att + i, vv);
-    }
-  }
-}
-
-// ------------------------------------------------------------------------------------------------ fused pass, lean
-// k_fused3: the fused single pass of k_fused (same arithmetic, same partition, same TMA ring) with a hot loop
-// written for issue efficiency -- the kernel is bound by the SM's issue slots and L1 data pipe, not by HBM
+// k_fused3 (the third version of this kernel; DESIGN.md §7 has the history) has a hot loop written for issue
+// efficiency -- the kernel is bound by the SM's issue slots and L1 data pipe, not by HBM
 // (DESIGN.md §7):
 //   * the loop is unrolled by two so the gather prefetch (group k+1) and the u_hat register queue alternate between
 //     two register sets instead of being copied every group;
@@ -931,26 +687,41 @@ constexpr int kF3Stage = kFRows * (kSlots * 8 + 16);  // 1664 B: 8 rows of value
 constexpr int kF3Bars = kFWarps * kFStages * 8;          // per stage: "full" mbarrier (TMA bytes)
 constexpr int kF3InstrMax = (kSmemMaxBytes - FRing::kBytes - kF3Bars - 1024) / 16 - 2;
 
-template <int KIND = R3_FUSED, int DIAG = 0>
+// Shared-slice regimes (SURVEY §8(d) sensitivity sweep): `zrep` copies of the CTA's z_instr accumulator (warp w
+// adds into copy w % zrep; more copies when the instrumental slice is small, fewer same-address CAS collisions);
+// SMATT: the attitude slice is small too (n_att <= kSmAttMax), so z_att is accumulated in `arep` shared-memory
+// copies (CAS) instead of L2 REDs, which serialise on few addresses.  Copies are summed once per CTA at the end.
+// IG: the instrumental slice is too large for shared memory: its gathers go through L1/L2 (__ldg) and its
+// contributions are L2 REDs (IdxRec then holds plain column offsets).  ZREP: zrep > 1 (a separate instantiation:
+// the runtime copy index costs ~4 % in the one-copy case).
+template <int KIND = R3_FUSED, int DIAG = 0, bool SMATT = false, bool IG = false, bool ZREP = false>
 __global__ void __launch_bounds__(kFWarps * 32, 1)
     k_fused3(SysView S, const double* __restrict__ x, double* __restrict__ u, double* __restrict__ zA,
              double* __restrict__ zsh, double* __restrict__ part, double* __restrict__ cpart,
              const DevState* __restrict__ st) {
   extern __shared__ __align__(128) unsigned char dsm[];
+  const int zrep = S.f3_zrep, arep = S.f3_arep;
   if (st->halted) return;
   constexpr bool kDot = KIND == R3_FUSED;  // computes the new u_hat (gathers, row dot, store, beta^2)
-  // shared memory: [ring | mbarriers | v_instr (slots) + v_glob | z_instr accumulator]
-  const int64_t nsl = S.ip.slots();
+  // shared memory: [ring | mbarriers | v_instr (slots) + v_glob | zrep x z_instr | arep x z_att (SMATT)]
+  const int64_t nsl = IG ? 0 : S.ip.slots(), zstride = IG ? 0 : nsl + 2;
   double* sh_x = reinterpret_cast<double*>(dsm + FRing::kBytes + kF3Bars);
-  double* sh_z = sh_x + nsl + 2;
+  double* sh_z = IG ? sh_x : sh_x + nsl + 2;  // IG: no instrumental arrays, z_att copies (SMATT) start here
+  double* sh_za = sh_z + zrep * zstride;
   for (int i = threadIdx.x; i < FRing::kBytes / 16; i += blockDim.x)
     reinterpret_cast<int4*>(dsm)[i] = make_int4(0, 0, 0, 0);
-  for (int64_t i = threadIdx.x; i < nsl; i += blockDim.x) {
-    sh_x[i] = 0.0;
-    sh_z[i] = 0.0;
+  constexpr bool kPlain = !SMATT && !IG && !ZREP;  // the C2-C5 regime (code kept as measured)
+  if (kPlain) {
+    for (int64_t i = threadIdx.x; i < nsl; i += blockDim.x) {
+      sh_x[i] = 0.0;
+      sh_z[i] = 0.0;
+    }
+  } else {
+    for (int64_t i = threadIdx.x; i < zstride * (1 + zrep) + (SMATT ? arep * S.n_att : 0); i += blockDim.x)
+      sh_x[i] = 0.0;
   }
   __syncthreads();
-  if (kDot) {
+  if (kDot && !IG) {
     for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) sh_x[S.ip.fwd(i)] = x[S.I0 + i];
     if (threadIdx.x == 0) sh_x[nsl] = S.n_glob ? x[S.G0] : 0.0;
   }
@@ -995,12 +766,15 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
   const double* xatt0 = x + S.A0 + j;
   const double* xatt1 = xatt0 + S.n_axis;
   const double* xatt2 = xatt1 + S.n_axis;
-  double* zatt0 = zsh + j;
+  double* zatt0 = (SMATT ? sh_za + (wid % arep) * S.n_att : zsh) + j;
   double* zatt1 = zatt0 + S.n_axis;
   double* zatt2 = zatt1 + S.n_axis;
+  double* const sh_zw = ZREP ? sh_z + (wid % zrep) * zstride : sh_z;  // this warp's z_instr copy
   const bool t5_ins = (j == 1 || j == 2);  // t=5 slot: lane 0 astro 4, lanes 1, 2 instr 4, 5, lane 3 global
   const int i5_shift = (j & 2) << 3;
-  const uint32_t i5_or = (j == 3) ? (uint32_t)nsl : 0u;  // lane 3 gathers v_glob (slot nsl); lane 0 ignores its g5
+  // lane 3 gathers v_glob (slot nsl; IG: column G0 = I0 + n_instr, which exists iff n_glob); lane 0 ignores its g5
+  const uint32_t i5_or = (j == 3) ? (IG ? (S.n_glob ? (uint32_t)S.n_instr : 0u) : (uint32_t)nsl) : 0u;
+  const double* const xins = x + S.I0;
   const int i4_shift = (j & 1) << 4;
   double* const urow = u + r_lo + r;
 
@@ -1056,8 +830,8 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
       P.g1 = (DIAG & 4) ? 0.5 : __ldg(xatt0 + P.k0);
       P.g2 = (DIAG & 4) ? 0.5 : __ldg(xatt1 + P.k0);
       P.g3 = (DIAG & 4) ? 0.5 : __ldg(xatt2 + P.k0);
-      P.g4 = (DIAG & 8) ? 0.5 : sh_x[P.i4];
-      P.g5 = (DIAG & 8) ? 0.5 : sh_x[P.i5];
+      P.g4 = (DIAG & 8) ? 0.5 : (IG ? __ldg(xins + P.i4) : sh_x[P.i4]);
+      P.g5 = (DIAG & 8) ? 0.5 : (IG ? __ldg(xins + P.i5) : sh_x[P.i5]);
     }
   };
 
@@ -1105,8 +879,9 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
       atomicAdd(zatt2 + P.k0, c3);
     }
     if (valid && !(DIAG & 1)) {
-      atomicAdd(sh_z + P.i4, c4v);
-      if (t5_ins) atomicAdd(sh_z + P.i5, c5);
+      double* const zi = IG ? zsh + S.n_att : sh_zw;
+      atomicAdd(zi + P.i4, c4v);
+      if (t5_ins) atomicAdd(zi + P.i5, c5);
     }
     if (!CHECK) {
       acc0 = fma(v[0], un, acc0);
@@ -1202,10 +977,25 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
     for (int q = 0; q < kFWarps; ++q) t += b2w[q];
     part[blockIdx.x] = t;
   }
-  for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
-    const double vv = sh_z[S.ip.fwd(i)];
-    if (vv != 0.0) atomicAdd(zsh + S.n_att + i, vv);
+  if (kPlain) {
+    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
+      const double vv = sh_z[S.ip.fwd(i)];
+      if (vv != 0.0) atomicAdd(zsh + S.n_att + i, vv);
+    }
+  } else if (!IG) {
+    for (int64_t i = threadIdx.x; i < S.n_instr; i += blockDim.x) {
+      const int64_t q = S.ip.fwd(i);
+      double vv = 0.0;
+      for (int c = 0; c < zrep; ++c) vv += sh_z[c * zstride + q];
+      if (vv != 0.0) atomicAdd(zsh + S.n_att + i, vv);
+    }
   }
+  if (SMATT)
+    for (int64_t i = threadIdx.x; i < S.n_att; i += blockDim.x) {
+      double vv = 0.0;
+      for (int c = 0; c < arep; ++c) vv += sh_za[c * S.n_att + i];
+      if (vv != 0.0) atomicAdd(zsh + i, vv);
+    }
 }
 
 // Fused mode, after k_beta: astro columns v' = (zA + constraint entries . u_hat_c) / beta - beta v  (P&S step b),
@@ -1817,31 +1607,58 @@ cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* p
   k_vshared<<<nblk, kRedThreads, 0, s>>>(S.n_sh, vsh, zsh, part, st, fused);
   return cudaGetLastError();
 }
+// Shared-memory plan of k_fused3: copies of the z_instr accumulator and, for small attitude slices, of z_att.
+struct F3Plan {
+  int zrep, arep;
+  size_t smem;
+};
+constexpr int64_t kSmAttMax = 4096;  // n_att up to this: z_att privatised in shared memory (L2 REDs contend below)
+static bool f3_ig(const SysView& S) { return S.ip.slots() > kF3InstrMax; }
+static F3Plan f3_plan(const SysView& S) {
+  const int64_t zb = f3_ig(S) ? 0 : 8 * (S.ip.slots() + 2), ab = 8 * S.n_att;
+  const int64_t fixed = FRing::kBytes + kF3Bars + zb;           // ring, mbarriers, v_instr
+  const int64_t avail = kSmemMaxBytes - 2048 - fixed;           // 2 KB: static shared memory of the kernel
+  F3Plan p{1, 0, 0};
+  if (S.n_att <= kSmAttMax && zb + ab <= avail) {
+    const int64_t r = std::min<int64_t>(kFWarps, avail / (zb + ab));
+    p.arep = (int)r;
+    p.zrep = zb ? (int)std::max<int64_t>(1, std::min<int64_t>(kFWarps, (avail - r * ab) / zb)) : 1;
+  } else {
+    p.zrep = zb ? (int)std::max<int64_t>(1, std::min<int64_t>(kFWarps, avail / zb)) : 1;
+  }
+  p.smem = (size_t)(fixed + (int64_t)p.zrep * zb + (int64_t)p.arep * ab);
+  return p;
+}
+template <int KIND, int DIAG, bool SMATT, bool IG, bool ZREP>
+static cudaError_t fz3v(const SysView& S, const F3Plan& P, int grid, const double* x, double* u, double* zA,
+                        double* zsh, double* part, double* cpart, const DevState* st, cudaStream_t s) {
+  static size_t attr_set = 0;
+  if (P.smem > attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(k_fused3<KIND, DIAG, SMATT, IG, ZREP>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)P.smem);
+    if (e != cudaSuccess) return e;
+    attr_set = P.smem;
+  }
+  SysView S2 = S;
+  S2.f3_zrep = P.zrep;
+  S2.f3_arep = P.arep;
+  k_fused3<KIND, DIAG, SMATT, IG, ZREP><<<grid, kFWarps * 32, P.smem, s>>>(S2, x, u, zA, zsh, part, cpart, st);
+  return cudaGetLastError();
+}
 template <int KIND, int DIAG>
 static cudaError_t fz3(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh, double* part,
                        double* cpart, const DevState* st, cudaStream_t s) {
-  const size_t smem = FRing::kBytes + kF3Bars + (2 * (size_t)S.ip.slots() + 4) * sizeof(double);
-  static size_t attr_set = 0;
-  if (smem > attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_fused3<KIND, DIAG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    attr_set = smem;
-  }
-  k_fused3<KIND, DIAG><<<grid, kFWarps * 32, smem, s>>>(S, x, u, zA, zsh, part, cpart, st);
-  return cudaGetLastError();
-}
-template <bool SM, int DIAG>
-static cudaError_t fz(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh, double* part,
-                      double* cpart, const DevState* st, cudaStream_t s) {
-  const size_t smem = FRing::kBytes + FRing::kBars + (SM ? (2 * (size_t)S.ip.slots() + 4) * sizeof(double) : 0);
-  static size_t attr_set = 0;  // dynamic shared memory opted in so far (static shared memory counts separately)
-  if (smem > attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_fused<SM, DIAG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    attr_set = smem;
-  }
-  k_fused<SM, DIAG><<<grid, kFWarps * 32, smem, s>>>(S, x, u, zA, zsh, part, cpart, st);
-  return cudaGetLastError();
+  const F3Plan P = f3_plan(S);
+  if (DIAG == 0 && f3_ig(S))
+    return P.arep > 0 ? fz3v<KIND, 0, true, true, false>(S, P, grid, x, u, zA, zsh, part, cpart, st, s)
+                      : fz3v<KIND, 0, false, true, false>(S, P, grid, x, u, zA, zsh, part, cpart, st, s);
+  if (DIAG == 0 && P.arep > 0) return fz3v<KIND, 0, true, false, true>(S, P, grid, x, u, zA, zsh, part, cpart, st, s);
+  if (DIAG == 0 && P.zrep > 1) return fz3v<KIND, 0, false, false, true>(S, P, grid, x, u, zA, zsh, part, cpart, st, s);
+  F3Plan Q = P;  // one z_instr copy, attitude REDs in L2 (the C2-C5 regime; DIAG experiments)
+  Q.smem -= (size_t)Q.arep * 8 * S.n_att + (size_t)(Q.zrep - 1) * 8 * (S.ip.slots() + 2);
+  Q.arep = 0;
+  Q.zrep = 1;
+  return fz3v<KIND, DIAG, false, false, false>(S, Q, grid, x, u, zA, zsh, part, cpart, st, s);
 }
 
 // Build-time experiment switch (not in the product build): compile with -DLSQR_DIAG_EXPERIMENTS to let the env var
@@ -1860,8 +1677,6 @@ static int diag_mode() {
 
 cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh,
                          double* part, double* cpart, const DevState* st, cudaStream_t s) {
-  // instrumental slice too large for shared memory: k_fused with instrumental gathers / REDs in global memory (L2)
-  if (S.ip.slots() > kF3InstrMax) return fz<false, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
 #ifdef LSQR_DIAG_EXPERIMENTS
   switch (diag_mode()) {
     case 1: return fz3<R3_FUSED, 1>(S, grid, x, u, zA, zsh, part, cpart, st, s);
@@ -1874,7 +1689,7 @@ cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u,
   return fz3<R3_FUSED, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
 }
 
-bool lean_products_ok(const SysView& S) { return S.ip.slots() <= kF3InstrMax; }
+bool lean_products_ok(const SysView&) { return true; }  // k_fused3 covers every instrumental-slice size (IG)
 cudaError_t launch_ap2_lean(const SysView& S, int grid, const double* u, double* zA, double* zsh, const DevState* st,
                             cudaStream_t s) {
   return fz3<R3_AP2, 0>(S, grid, nullptr, const_cast<double*>(u), zA, zsh, nullptr, nullptr, st, s);

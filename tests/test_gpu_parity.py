@@ -369,12 +369,21 @@ def test_set_system_roundtrip_and_validation(avu):
     s.close()
 
 
-@pytest.mark.parametrize("case", ["instr_global", "empty_stars", "noglob"])
+@pytest.mark.parametrize("case", ["instr_global", "instr_global_att_l2", "instr_copies_att_l2", "empty_stars",
+                                  "noglob"])
 def test_lsqr_fused_edge_cases(avu, case):
     """Fused and two-pass iterations on the paths the default configs do not exercise: the instrumental slice too
-    large for shared memory (global-memory gathers/REDs), stars with no observations, no global column."""
+    large for shared memory (global-memory gathers/REDs) with a small (shared-memory) or larger (L2 REDs) attitude
+    slice, several z_instr copies with L2 attitude REDs, stars with no observations, no global column.  (C1 itself
+    runs the small-attitude + z_instr-copies regime, C2 the one-copy / L2-attitude regime.)"""
     if case == "instr_global":  # 120k rows x 30.2k columns (overdetermined), instrumental slice 192 KB
         w = W.C1.replace(name="C1i", n_instr=24_000, n_obs=120_000)
+        counts = None
+    elif case == "instr_global_att_l2":  # as above with n_att above the shared-memory attitude limit (4,096)
+        w = W.C1.replace(name="C1ia", n_att=4_200, n_instr=24_000, n_obs=120_000)
+        counts = None
+    elif case == "instr_copies_att_l2":  # n_instr = 60 (16 z_instr copies), attitude by L2 REDs
+        w = W.C1.replace(name="C1ra", n_att=4_200)
         counts = None
     elif case == "empty_stars":
         w = W.micro(n_stars=50, obs=12, n_ext=6, seed=17)
