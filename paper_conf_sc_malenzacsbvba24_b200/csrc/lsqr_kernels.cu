@@ -661,8 +661,7 @@ using FRing = RingT<kFRows, kFStages, kFWarps>;
 constexpr int kSmemMaxBytes = 232448;  // 227 KB opt-in per CTA on sm_100
 
 // k_fused3 (the third version of this kernel; DESIGN.md §7 has the history) has a hot loop written for issue
-// efficiency -- the kernel is bound by the SM's issue slots and L1 data pipe, not by HBM
-// (DESIGN.md §7):
+// efficiency -- the kernel is bound by the SM's issue slots and L1 data pipe, not by HBM:
 //   * the loop is unrolled by two so the gather prefetch (group k+1) and the u_hat register queue alternate between
 //     two register sets instead of being copied every group;
 //   * the ring's shared memory is zeroed at entry, so the index records of rows past the end of a warp's range are
@@ -671,9 +670,8 @@ constexpr int kSmemMaxBytes = 232448;  // 227 KB opt-in per CTA on sm_100
 //     accumulator `acc5`, folded per star (lane 0: zA, lane 3: global sum; lanes 1, 2 discard theirs);
 //   * shared-memory FP64 accumulation of the instrumental slice uses the compiler's CAS-spin loop (ATOMS.CAST.SPIN;
 //     measured faster than an explicit atom.cas loop);
-//   * no proxy fence before re-filling a stage: lane 0 issues the TMA that overwrites a stage only after every lane
-//     has USED the values it loaded from it (the row dot depends on all of them; __syncwarp), so no read of the
-//     stage is outstanding; the fence cost a MEMBAR.ALL.CTA per group.
+//   * one proxy fence per two stages: lane 0 re-fills two released slots after one fence.async (generic-proxy reads
+//     of a slot before the async-proxy TMA write into it; without the fence the full-size C2 parity test fails).
 //
 // The same loop, templated on KIND, is also the two-pass iteration's aprod2 (the paper's structure: A read twice per
 // iteration):
@@ -693,7 +691,7 @@ constexpr int kF3InstrMax = (kSmemMaxBytes - FRing::kBytes - kF3Bars - 1024) / 1
 // copies (CAS) instead of L2 REDs, which serialise on few addresses.  Copies are summed once per CTA at the end.
 // IG: the instrumental slice is too large for shared memory: its gathers go through L1/L2 (__ldg) and its
 // contributions are L2 REDs (IdxRec then holds plain column offsets).  ZREP: zrep > 1 (a separate instantiation:
-// the runtime copy index costs ~4 % in the one-copy case).
+// in the one-copy case the runtime copy index changed the schedule and measured 2-4 % slower).
 template <int KIND = R3_FUSED, int DIAG = 0, bool SMATT = false, bool IG = false, bool ZREP = false>
 __global__ void __launch_bounds__(kFWarps * 32, 1)
     k_fused3(SysView S, const double* __restrict__ x, double* __restrict__ u, double* __restrict__ zA,
