@@ -1,5 +1,6 @@
 """Small end-to-end run used under compute-sanitizer (tests/test_sanitizer.py): generate, precondition, products,
-two solves (fused and two-pass), set_system round trip, and the bitwise-reproducible mode (NEXT-4).  Exits non-zero on any library error."""
+two solves (fused and two-pass) in each shared-slice regime of the fused kernel, set_system round trip, and the
+bitwise-reproducible mode (NEXT-4).  Exits non-zero on any library error."""
 import os
 import sys
 
@@ -28,6 +29,16 @@ def main():
         s.set_system(g["vals"], g["mA"], g["mT"], g["iC"], g["b"])
         out = s.solve(itn_limit=3, fused=fused, use_graph=True)
         s.close()
+    # the other shared-slice regimes of the fused kernel: one z_instr copy + L2 attitude REDs (the C2-C5 regime),
+    # and the instrumental slice in L1/L2 (IG) with L2 attitude REDs
+    for w2 in (W.C1.replace(name="san-plain", n_stars=300, n_obs=6000, n_att=6_000, n_instr=6_000),
+               W.C1.replace(name="san-ig", n_stars=300, n_obs=6000, n_att=6_000, n_instr=24_000)):
+        for fused in (True, False):
+            s = avu.Solver.synthetic(w2, torch_alloc=False)
+            s.precondition()
+            out = s.solve(itn_limit=4, atol=0, btol=0, conlim=0, fixed_count=True, fused=fused, use_graph=False)
+            assert out["itn"] == 4 and np.isfinite(out["x"]).all()
+            s.close()
     s = avu.Solver.synthetic(w, torch_alloc=False)
     s.set_reproducible(True)
     s.precondition()
