@@ -390,7 +390,8 @@ def run_ours(args):
     }
     s.close()
     if rank == 0 and n == 1 and args.cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline(base, iters=args.cpu_iters, repro=args.repro)
+        line["cpu_baseline"] = cpu_baseline(base, iters=min(args.cpu_iters, 5) if args.repro else args.cpu_iters,
+                                            repro=args.repro)
     if rank == 0:
         emit(line)
     if multi:
@@ -429,7 +430,8 @@ def main():
     ap.add_argument("--config", default="C2", choices=sorted(W.CONFIGS))
     ap.add_argument("--no-e2e", dest="e2e", action="store_false")
     ap.add_argument("--no-cpu-baseline", dest="cpu_baseline", action="store_false")
-    ap.add_argument("--cpu-iters", type=int, default=3)
+    ap.add_argument("--cpu-iters", type=int, default=30,
+                    help="oracle LSQR iterations timed for cpu_baseline (a bounded sample: ~10 s of CPU work at C2)")
     ap.add_argument("--n-att", type=int, default=0, help="override n_att (multiple of 3, >= 12; sensitivity sweep)")
     ap.add_argument("--n-instr", type=int, default=0, help="override n_instr (multiple of 6; sensitivity sweep)")
     ap.add_argument("--fused", dest="fused", action="store_true", default=True,
