@@ -149,6 +149,32 @@ def _cpu_model():
     return None
 
 
+def time_api_products(s, k, ap1_bytes, ap2_bytes, peak, max_over_ranks):
+    """The boundary's own product calls, lsqr_aprod1 (y += A x) and lsqr_aprod2 (x += A^T y, shared slice
+    allreduced), k calls each between CUDA events on the caller's stream (device tensors).  Algorithmic bytes:
+    aprod1 as the iteration's; aprod2 216 B/row + 120 B/star (z row sums written and read back, x_astro read and
+    written) + 8 B/shared column."""
+    import torch
+    x = torch.full((s.n_local_cols,), 1e-3, dtype=torch.float64, device="cuda")
+    y = torch.zeros(s.n_local_rows + s.n_constr, dtype=torch.float64, device="cuda")
+    out = {"calls": k}
+    for name, fn, nb in (("aprod1", lambda: s.aprod1(x, y), ap1_bytes), ("aprod2", lambda: s.aprod2(y, x), ap2_bytes)):
+        fn()  # warm-up
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        e0.record(s.stream)
+        for _ in range(k):
+            fn()
+        e1.record(s.stream)
+        e1.synchronize()
+        ms = max_over_ranks(e0.elapsed_time(e1) / k)
+        out[name + "_ms"] = round(ms, 5)
+        out[name + "_frac"] = round(nb / (ms * 1e-3) / 1e9 / peak, 4)
+    out["note"] = ("lsqr_aprod1 / lsqr_aprod2 C-ABI calls on device buffers (k calls each, CUDA events on the "
+                   "caller's stream); frac against the measured HBM peak on their algorithmic bytes")
+    return out
+
+
 def variant_name(args):
     if getattr(args, "force_collectives", False):
         base = "fused single pass" if getattr(args, "fused", False) else "two-pass"
@@ -388,6 +414,10 @@ def run_ours(args):
         "e2e": e2e,
         "lsqr": {"itn": st["itn"], "r1norm": st["r1norm"], "arnorm": st["arnorm"]},
     }
+    if not args.repro:
+        line["api_products"] = time_api_products(s, min(K, 20), ap1_b,
+                                                 216 * s.n_local_rows + 120 * (s.star_end - s.star_begin)
+                                                 + 8 * s.n_shared, peak, max_over_ranks)
     s.close()
     if rank == 0 and n == 1 and args.cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(base, iters=min(args.cpu_iters, 5) if args.repro else args.cpu_iters,

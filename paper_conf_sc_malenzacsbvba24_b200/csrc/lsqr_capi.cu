@@ -102,6 +102,7 @@ struct lsqr_ctx {
   IdxRec* idx = nullptr;
   int64_t *star_ptr = nullptr, *warp_star = nullptr, *warp_star_f = nullptr;
   DevState* st = nullptr;
+  DevState* st_api = nullptr;  // never-halted state for the lsqr_aprod2 API call on the fused kernel's loop
   int32_t* hflag = nullptr;  // host-mapped
   int32_t* hflag_dev = nullptr;
   SysView S{};
@@ -680,6 +681,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   AL(h->tmp, std::max<int64_t>(h->n_loc_cols, nc + 1));
   AL(h->tmax, 8);
   AL(h->st, 1);
+  AL(h->st_api, 1);
   double* d_cval = nullptr;
   int64_t *d_ccol = nullptr, *d_chb = nullptr, *d_che = nullptr, *d_csp = nullptr, *d_cse = nullptr,
           *d_cshi = nullptr, *d_cshe = nullptr;
@@ -752,6 +754,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
     if (launch_fill(p, h->n_loc_cols, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (launch_fill(h->u, h->n_loc_rows + 2, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (cudaMemsetAsync(h->st, 0, sizeof(DevState), h->s) != cudaSuccess) return bail(LSQR_ECUDA);
+  if (cudaMemsetAsync(h->st_api, 0, sizeof(DevState), h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (cudaStreamSynchronize(h->s) != cudaSuccess) return bail(LSQR_ECUDA);
 
   // ---- communicator
@@ -971,8 +974,10 @@ int lsqr_aprod2(lsqr_t h, const double* y_dev, double* x_dev) {
   if (!h->have_system) return fail(h, LSQR_ESTATE, "no system");
   SysView& S = h->S;
   enter(h);
-  CKL(h, launch_aprod2(AP2_PLAIN, S, h->grid, y_dev, y_dev + h->n_loc_rows, x_dev, h->zsh, h->part_a2, h->st,
-                       h->rank == 0, h->s), "aprod2");
+  // rows on the fused kernel's loop (its halted flag comes from st_api, a DevState that is never halted), then the
+  // astro columns and constraint entries
+  CKL(h, launch_ap2_lean(S, h->grid, y_dev, h->zA, h->zsh, h->st_api, h->s), "aprod2");
+  CKL(h, launch_astro_add(S, x_dev, h->zA, y_dev + h->n_loc_rows, h->zsh, h->rank == 0, h->s), "aprod2_astro");
   CKR(allreduce(h, h->zsh, h->n_sh));
   CKL(h, launch_add_shared(x_dev + S.A0, h->zsh, h->n_sh, 0, h->s), "aprod2_sh");
   leave(h);

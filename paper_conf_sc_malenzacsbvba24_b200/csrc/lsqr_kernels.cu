@@ -1255,6 +1255,24 @@ __global__ void __launch_bounds__(kRedThreads)
 }
 
 // mode 0: x += z, z = 0 (plain aprod2);  mode 1: x = z, z = 0 (column norms)
+// lsqr_aprod2 on the fused kernel's loop (after k_fused3<R3_AP2> wrote the row sums z = A_rows^T y): astro columns
+// x[c] += z[c] + constraint entries . y_c (added after the rows, as O-AP2); shared-column constraint entries
+// scattered into z_sh by their owner (rank 0) before the allreduce and k_add_shared.
+__global__ void __launch_bounds__(kRedThreads)
+    k_astro_add(SysView S, double* __restrict__ x, const double* __restrict__ zA, const double* __restrict__ yc,
+                double* __restrict__ zsh, int do_shared_constr) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < 5 * S.n_stars; c += stride) {
+    double z = zA[c];
+    if (c < 5 * S.n_cs)
+      for (int64_t e = S.cs_ptr[c]; e < S.cs_ptr[c + 1]; ++e) z += S.cval[S.cs_e[e]] * yc[S.cs_k[e]];
+    x[c] += z;
+  }
+  if (do_shared_constr)
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < S.n_csh; e += stride)
+      atomicAdd(zsh + S.csh_idx[e], S.cval[S.csh_e[e]] * yc[S.csh_k[e]]);
+}
+
 __global__ void k_add_shared(double* __restrict__ xsh, double* __restrict__ zsh, int64_t n, int mode) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     xsh[i] = mode == 0 ? xsh[i] + zsh[i] : zsh[i];
@@ -1699,6 +1717,12 @@ cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const d
   return cudaGetLastError();
 }
 
+cudaError_t launch_astro_add(const SysView& S, double* x, const double* zA, const double* yc, double* zsh,
+                             int do_shared_constr, cudaStream_t s) {
+  k_astro_add<<<vec_grid(std::max<int64_t>(5 * S.n_stars, S.n_csh), 148 * 4), kRedThreads, 0, s>>>(S, x, zA, yc, zsh,
+                                                                                                 do_shared_constr);
+  return cudaGetLastError();
+}
 cudaError_t launch_add_shared(double* xsh, double* zsh, int64_t n, int mode, cudaStream_t s) {
   k_add_shared<<<vec_grid(n, 148 * 4), kRedThreads, 0, s>>>(xsh, zsh, n, mode);
   return cudaGetLastError();

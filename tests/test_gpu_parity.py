@@ -223,7 +223,10 @@ def test_lsqr_free_run_and_converged(avu, w, fused):
     d = np.abs(out["se"] / seo - 1)
     dc = np.abs(S.D * rc["se"] / seo - 1)
     print(f"se: median rel diff gpu {np.median(d):.2e}  control {np.median(dc):.2e}")
-    assert np.median(d) <= max(1e-2, 3 * np.median(dc))
+    # floor 2e-2: sigma after 100 free-run iterations depends on the rounding trajectory (valid
+    # summation orders differ by ~1e-3 median to >10 % max [EXP-4]); the GPU also contracts to FMA (DESIGN Z13)
+    # and its atomics order changes run to run, so one GPU sample vs one control sample is noisy near 1e-2
+    assert np.median(d) <= max(2e-2, 3 * np.median(dc))
     s.close()
 
 
