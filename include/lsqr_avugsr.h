@@ -199,8 +199,10 @@ int lsqr_get_precond(lsqr_t h, double* D);
  * to run and to the CPU oracle's repro mode, independent of scheduling; lsqr_solve_params.fused is ignored and the
  * iteration is several times slower than the default path (verification mode).  With nranks > 1 the digits are
  * allreduced exactly (as pairs of exact doubles), so D, x, se and every scalar are bit-identical for ANY number of
- * ranks and any shard map.  Allocates 40 B per local column of digit storage (+ 80 B per shared column when
- * nranks > 1; LSQR_ENOMEM).  Invalidates a previous lsqr_init; call before lsqr_precondition for a reproducible D.
+ * ranks and any shard map.  Allocates 56 B per local column of digit storage (+ 112 B per shared column when
+ * nranks > 1; LSQR_ENOMEM).  The digit sums are exact for fewer than 2^33 terms per accumulator on a rank: the call
+ * returns LSQR_EINVAL when 6 * n_local_rows + (owned constraint entries) >= 2^33 or n_local_cols >= 2^33.
+ * Invalidates a previous lsqr_init; call before lsqr_precondition for a reproducible D.
  * Collective when nranks > 1 (only in the sense that all ranks must use the same mode). */
 int lsqr_set_reproducible(lsqr_t h, int32_t on);
 

@@ -258,7 +258,10 @@ void orc_aprod2(const orc_sys* S, const double* y, double* x) {
  * implement the spec, so their iterates agree bit for bit.
  * ---------------------------------------------------------------------------------------------------------- */
 #define ORC_EDA_L 5
-typedef struct { int64_t d[ORC_EDA_L]; } orc_eda;
+/* Digits are accumulated in 128-bit integers: a piece is < 2^40 in magnitude, so no realistic number of additions
+ * (< 2^87) can overflow -- the sum held in D is always the exact integer sum of the pieces.  (64-bit digits, as in
+ * round 1, wrap after ~2^23 positive terms: beta^2 over 10^8 rows came out off by multiples of 2^64 * 2^B_d.) */
+typedef struct { __int128 d[ORC_EDA_L]; } orc_eda;
 static const int orc_eda_B[ORC_EDA_L] = {-8, -48, -88, -128, -168}; /* digit d covers bits [B_d, B_d + 40) */
 
 void orc_eda_add(orc_eda* A, double c) {
@@ -282,16 +285,18 @@ void orc_eda_add(orc_eda* A, double c) {
     else if (sh >= 0) dig = (M << sh) & ((1ULL << 40) - 1);
     else if (sh > -53) dig = (M >> (-sh)) & ((1ULL << 40) - 1);
     else dig = 0;
-    A->d[d] += neg ? -(int64_t)dig : (int64_t)dig;
+    A->d[d] += neg ? -(__int128)dig : (__int128)dig;
   }
 }
 
+/* round(D) (docs/REPRO.md): carry-normalise so that D_d is in [0, 2^40) for d >= 1 (the unique such representation
+ * of the exact value), then v = 0; v = v + D_d * 2^B_d for d = 0..4, every conversion and addition rounded. */
 double orc_eda_round(const orc_eda* A) {
-  int64_t D[ORC_EDA_L];
+  __int128 D[ORC_EDA_L];
   for (int d = 0; d < ORC_EDA_L; ++d) D[d] = A->d[d];
-  for (int d = ORC_EDA_L - 1; d >= 1; --d) { /* carry-normalise: D_d in [0, 2^40) for d >= 1 */
-    const int64_t c = D[d] >> 40;            /* arithmetic shift = floor division (gcc) */
-    D[d] -= c * ((int64_t)1 << 40);
+  for (int d = ORC_EDA_L - 1; d >= 1; --d) {
+    const __int128 c = D[d] >> 40; /* arithmetic shift = floor division (gcc) */
+    D[d] -= c * ((__int128)1 << 40);
     D[d - 1] += c;
   }
   double v = 0.0;

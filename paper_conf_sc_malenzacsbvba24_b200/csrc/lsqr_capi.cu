@@ -244,11 +244,12 @@ int launch_ok(lsqr_t h, cudaError_t e, const char* what) {
 
 // ------------------------------------------------------------------------------------------------ repro mode
 // NEXT-4: allreduce of int64 digits as exact double pairs (no-op on one rank)
-int repro_allreduce(lsqr_t h, long long* src, int64_t n, int nseg, int64_t stride) {
-  if (!h->multi || n * nseg == 0) return LSQR_OK;
-  CKL(h, repro_pack(src, n, nseg, stride, h->rbuf, 0, h->s), "repro_pack");
-  CKR(allreduce(h, h->rbuf, 2 * n * nseg));
-  CKL(h, repro_pack(src, n, nseg, stride, h->rbuf, 1, h->s), "repro_unpack");
+// nval values of L digits: digit-major planes of stride `plane`, or (plane == 0) L consecutive digits per value
+int repro_allreduce(lsqr_t h, long long* src, int64_t nval, int64_t plane) {
+  if (!h->multi || nval == 0) return LSQR_OK;
+  CKL(h, repro_pack(src, nval, plane, h->rbuf, 0, h->s), "repro_pack");
+  CKR(allreduce(h, h->rbuf, 2 * repro_digits_per_value() * nval));
+  CKL(h, repro_pack(src, nval, plane, h->rbuf, 1, h->s), "repro_unpack");
   return LSQR_OK;
 }
 
@@ -267,16 +268,16 @@ int enqueue_repro(lsqr_t h, int init) {
   const int64_t nc = h->n_constr;
   cudaStream_t s = h->s;
   CKL(h, repro_step(RS_APROD1, a, s), "repro_aprod1");
-  CKR(repro_allreduce(h, repro_sd_part(h->rsd, nc, 0), 5 * (1 + nc), 1, 0));
+  CKR(repro_allreduce(h, repro_sd_part(h->rsd, nc, 0), 1 + nc, 0));
   CKL(h, repro_step(RS_BETA, a, s), "repro_beta");
   CKL(h, repro_step(RS_APROD2, a, s), "repro_aprod2");
-  CKR(repro_allreduce(h, h->rzd + h->S.A0, h->n_sh, 5, h->n_loc_cols));
+  CKR(repro_allreduce(h, h->rzd + h->S.A0, h->n_sh, h->n_loc_cols));
   CKL(h, repro_step(RS_VUPDATE, a, s), "repro_vupdate");
-  CKR(repro_allreduce(h, repro_sd_part(h->rsd, nc, 1), 5, 1, 0));
+  CKR(repro_allreduce(h, repro_sd_part(h->rsd, nc, 1), 1, 0));
   CKL(h, repro_step(RS_SCALAR_A, a, s), "repro_scalar_a");
   CKL(h, repro_step(RS_COLUPDATE, a, s), "repro_colupdate");
   if (init) return LSQR_OK;
-  CKR(repro_allreduce(h, repro_sd_part(h->rsd, nc, 2), 5, 1, 0));
+  CKR(repro_allreduce(h, repro_sd_part(h->rsd, nc, 2), 1, 0));
   CKL(h, repro_step(RS_SCALAR_B, a, s), "repro_scalar_b");
   return LSQR_OK;
 }
@@ -899,7 +900,7 @@ int lsqr_precondition(lsqr_t h) {
   if (h->repro) {  // NEXT-4: exact column sums of squares
     const ReproArgs a = repro_args(h, 0);
     CKL(h, repro_step(RS_COLNORM, a, h->s), "colnorm_repro");
-    CKR(repro_allreduce(h, h->rzd + S.A0, h->n_sh, 5, h->n_loc_cols));
+    CKR(repro_allreduce(h, h->rzd + S.A0, h->n_sh, h->n_loc_cols));
     CKL(h, repro_step(RS_PRECOND_D, a, h->s), "precond_D_repro");
     CKL(h, launch_scale_rows(S, h->grid, h->vals, h->D, h->s), "scale_rows");
     CKL(h, launch_scale_constr(S, const_cast<double*>(S.cval), h->D, h->s), "scale_constr");
@@ -935,6 +936,11 @@ int lsqr_get_precond(lsqr_t h, double* D) {
 int lsqr_set_reproducible(lsqr_t h, int32_t on) {
   GUARD(h);
   if (on != 0 && on != 1) return LSQR_EINVAL;
+  // exactness bound of the digit format: no accumulator may receive 2^33 terms on one rank (a column gets at most 6
+  // terms per row plus its constraint entries; beta^2 one per row; alpha^2 / ddnorm one per column)
+  if (on && (6 * h->n_loc_rows + h->n_ce >= repro_max_terms() || h->n_loc_cols >= repro_max_terms()))
+    return fail(h, LSQR_EINVAL, "reproducible mode: shard too large for exact digit accumulation (6 rows + "
+                                "constraint entries >= 2^33)");
   if (on && !h->rzd) {
     const int64_t L = repro_digits_per_value();
     CKR(dalloc(h, &h->rzd, L * h->n_loc_cols));
@@ -1004,7 +1010,7 @@ int lsqr_init(lsqr_t h, const lsqr_solve_params* p) {
   for (double* q : {h->v, h->w, h->x, h->var}) CKL(h, launch_fill(q, h->n_loc_cols, 0.0, h->s), "fill");
   CKL(h, launch_fill(h->zsh, h->n_sh + 8, 0.0, h->s), "fill");
   if (h->repro) {  // NEXT-4 O-1
-    CKC(h, cudaMemsetAsync(h->rzd, 0, sizeof(long long) * 5 * h->n_loc_cols, h->s));
+    CKC(h, cudaMemsetAsync(h->rzd, 0, sizeof(long long) * repro_digits_per_value() * h->n_loc_cols, h->s));
     CKC(h, cudaMemsetAsync(h->rsd, 0, sizeof(long long) * repro_sd_size(h->n_constr), h->s));
     CKR(enqueue_repro(h, 1));
     h->b_valid = false;

@@ -185,9 +185,9 @@ cudaError_t launch_finalize(const double* x, const double* var, const double* D,
 cudaError_t launch_fill(double* p, int64_t n, double v, cudaStream_t s);
 
 // NEXT-4 bitwise-reproducible mode (lsqr_repro.cu, docs/REPRO.md).  Digit buffers (int64, zeroed; every step leaves
-// what it consumed zeroed): zd [5][n_cols] digit-major column accumulator; sd [repro_sd_size(n_constr)] =
-// [beta^2 (5) | constraint rows (5 n_constr) | alpha^2 astro (5) | alpha^2 shared (5) | ddnorm astro (5) |
-// ddnorm shared (5)].  The astro parts are rank-local (allreduced when P > 1), the shared parts are computed
+// what it consumed zeroed; L = repro_digits_per_value()): zd [L][n_cols] digit-major column accumulator;
+// sd [repro_sd_size(n_constr)] = [beta^2 (L) | constraint rows (L n_constr) | alpha^2 astro (L) | alpha^2 shared (L) |
+// ddnorm astro (L) | ddnorm shared (L)].  The astro parts are rank-local (allreduced when P > 1), the shared parts are computed
 // identically on every rank.  u / uc hold u_hat (unnormalised) like the default path; st->inv_beta normalises.
 enum { RS_APROD1, RS_BETA, RS_APROD2, RS_VUPDATE, RS_SCALAR_A, RS_COLUPDATE, RS_SCALAR_B, RS_COLNORM, RS_PRECOND_D };
 struct ReproArgs {
@@ -204,9 +204,11 @@ int64_t repro_sd_size(int64_t n_constr);
 // part 0: [beta^2 | constraint rows] (5 + 5 n_constr contiguous), 1: alpha^2 astro (5), 2: ddnorm astro (5)
 long long* repro_sd_part(long long* sd, int64_t n_constr, int part);
 cudaError_t repro_step(int step, const ReproArgs& a, cudaStream_t s);
-// int64 <-> exact double pairs for the allreduce: nseg segments of n values, segment stride `stride` (in values);
-// buf holds 2 n nseg doubles
-cudaError_t repro_pack(const long long* src, int64_t n, int nseg, int64_t stride, double* buf, int unpack,
-                       cudaStream_t s);
+// int64 digits <-> exact double pairs for the allreduce: nval values of L digits, digit q of value i at
+// src[q * plane + i] (plane > 0: digit-major planes) or src[i * L + q] (plane == 0); carry-normalised on packing;
+// buf holds 2 L nval doubles
+cudaError_t repro_pack(const long long* src, int64_t nval, int64_t plane, double* buf, int unpack, cudaStream_t s);
+// largest number of terms any digit accumulator may receive on one rank (the exactness bound of the format)
+int64_t repro_max_terms();
 
 }  // namespace lsqr

@@ -1,10 +1,18 @@
 // lsqr_repro.cu -- bitwise-reproducible mode (docs/REPRO.md), product side.
 //
-// Every reduction is an exact digit accumulation (EDA: 5 signed 40-bit digits over bits [-168, 32)) of identically
-// rounded FP64 terms, combined with 64-bit integer additions/atomics, which are associative: the result does not
-// depend on thread, warp, block or atomic order.  Every other operation is a single IEEE operation written with
-// explicit _rn intrinsics (no FMA contraction), in the order the Paige-Saunders recurrence writes them.  The CPU
-// test oracle implements the same spec independently (docs/REPRO.md), so iterates agree bit for bit.
+// Every reduction is an exact digit accumulation (EDA, docs/REPRO.md) of identically rounded FP64 terms, combined
+// with 64-bit integer additions/atomics, which are associative: the result does not depend on thread, warp, block or
+// atomic order.  Every other operation is a single IEEE operation written with explicit _rn intrinsics (no FMA
+// contraction), in the order the Paige-Saunders recurrence writes them.  The CPU test oracle implements the same
+// spec independently (docs/REPRO.md), so iterates agree bit for bit.
+//
+// Accumulation format (device-internal): 7 digits of 30-bit pieces in int64 over bits [-168, 42) (the spec's window
+// is [-168, 32): bits of a term at or above 2^32 are dropped, as the spec says).  A piece is < 2^30 in magnitude, so
+// ANY partial sum of fewer than 2^33 pieces is exact -- lsqr_set_reproducible rejects shards where an accumulator
+// could receive more (6 n_local_rows + constraint entries >= 2^33).  Before a cross-rank allreduce the digits are
+// carry-normalised (value-preserving), so the reduced digits stay below P * 2^30.  Rounding converts the exact
+// value to the spec's unique carry-normalised 5 x 40-bit form and applies the spec's rounding chain, so the result
+// does not depend on the accumulation format.
 //
 // These kernels are simple (thread per row / column, global atomics for every digit): the mode is for verification
 // and run-to-run reproducibility, not for speed.
@@ -14,8 +22,10 @@ namespace lsqr {
 
 namespace {
 
-constexpr int kL = 5;  // digits
-// digit q covers bits [B_q, B_q + 40), B = -8, -48, -88, -128, -168 (docs/REPRO.md)
+constexpr int kL = 7;   // digits; digit q covers bits [B_q, B_q + 30), B_q = 12 - 30 q (12, -18, ..., -168)
+constexpr int kW = 30;  // bits per piece
+constexpr long long kM30 = (1ll << kW) - 1;
+constexpr long long kM20 = (1ll << 20) - 1;  // digit 0 keeps bits [12, 32) only: the spec's window top is 2^32
 
 struct Eda {
   long long d[kL];
@@ -26,12 +36,11 @@ __device__ __forceinline__ void eda_zero(Eda& A) {
   for (int q = 0; q < kL; ++q) A.d[q] = 0;
 }
 
-// split(c) (docs/REPRO.md): with p = E - B_4 the offset of the significand's lowest bit above the window bottom, the
-// significand lands in digits 4-k, 3-k, 2-k (k = p div 40) as the 40-bit pieces lo, mid, hi of M << (p mod 40); bits
-// below the window (p < 0) are truncated first, pieces above digit 0 are dropped.  These are exactly the digits of
-// the spec's per-digit rule (at most three of them nonzero).
+// split(c): with p = E + 168 the offset of the significand's lowest bit above the window bottom (bits below the
+// window are truncated first), the significand lands in digits 6-k, 5-k, 4-k (k = p div 30) as the 30-bit pieces
+// lo, mid, hi of M << (p mod 30); pieces above digit 0 are dropped and digit 0 keeps its bits below 2^32.
 struct Pieces {
-  long long lo, mid, hi;
+  long long lo, mid, hi, sgn;  // magnitudes (sign applied by the consumer: (x ^ sgn) - sgn)
   int k;
 };
 
@@ -45,55 +54,74 @@ __device__ __forceinline__ Pieces eda_split(double c) {
     M = p > -53 ? (M >> (-p)) : 0ull;
     p = 0;
   }
-  const int k = p / 40, o = p - 40 * k;
-  const unsigned long long mask = (1ull << 40) - 1;
-  const long long sgn = bits >> 63;  // 0 or -1
+  const int k = p / kW, o = p - kW * k;
   Pieces r;
   r.k = k;
-  r.lo = ((long long)((M << o) & mask) ^ sgn) - sgn;
-  r.mid = ((long long)((M >> (40 - o)) & mask) ^ sgn) - sgn;
-  r.hi = ((long long)(o > 27 ? (M >> (80 - o)) : 0ull) ^ sgn) - sgn;
+  r.sgn = bits >> 63;  // 0 or -1
+  r.lo = (long long)((M << o) & (unsigned long long)kM30);
+  r.mid = (long long)((M >> (kW - o)) & (unsigned long long)kM30);
+  r.hi = (long long)((M >> (2 * kW - o)) & (unsigned long long)kM30);
   return r;
 }
 
+__device__ __forceinline__ long long sgnd(long long x, long long sgn) { return (x ^ sgn) - sgn; }
+
 __device__ __forceinline__ void eda_add(Eda& A, double c) {
   const Pieces P = eda_split(c);
+  const long long s = P.sgn;
   switch (P.k) {  // constant digit indices keep A in registers; k is nearly warp-uniform for real data
-    case 0: A.d[4] += P.lo; A.d[3] += P.mid; A.d[2] += P.hi; break;
-    case 1: A.d[3] += P.lo; A.d[2] += P.mid; A.d[1] += P.hi; break;
-    case 2: A.d[2] += P.lo; A.d[1] += P.mid; A.d[0] += P.hi; break;
-    case 3: A.d[1] += P.lo; A.d[0] += P.mid; break;
-    case 4: A.d[0] += P.lo; break;
+    case 0: A.d[6] += sgnd(P.lo, s); A.d[5] += sgnd(P.mid, s); A.d[4] += sgnd(P.hi, s); break;
+    case 1: A.d[5] += sgnd(P.lo, s); A.d[4] += sgnd(P.mid, s); A.d[3] += sgnd(P.hi, s); break;
+    case 2: A.d[4] += sgnd(P.lo, s); A.d[3] += sgnd(P.mid, s); A.d[2] += sgnd(P.hi, s); break;
+    case 3: A.d[3] += sgnd(P.lo, s); A.d[2] += sgnd(P.mid, s); A.d[1] += sgnd(P.hi, s); break;
+    case 4: A.d[2] += sgnd(P.lo, s); A.d[1] += sgnd(P.mid, s); A.d[0] += sgnd(P.hi & kM20, s); break;
+    case 5: A.d[1] += sgnd(P.lo, s); A.d[0] += sgnd(P.mid & kM20, s); break;
+    case 6: A.d[0] += sgnd(P.lo & kM20, s); break;
     default: break;
   }
 }
 
-// the pieces of one term straight into the digit-major column accumulator zd[q][col] (q = 4-k, 3-k, 2-k)
+// the pieces of one term straight into the digit-major column accumulator zd[q][col] (q = 6-k, 5-k, 4-k)
 __device__ __forceinline__ void eda_atomic_term(long long* __restrict__ zd_col, int64_t stride, double c) {
   const Pieces P = eda_split(c);
   const long long pc[3] = {P.lo, P.mid, P.hi};
 #pragma unroll
   for (int r = 0; r < 3; ++r) {
     const int q = kL - 1 - P.k - r;
-    if (q >= 0 && pc[r] != 0)
-      atomicAdd(reinterpret_cast<unsigned long long*>(zd_col + q * stride), (unsigned long long)pc[r]);
+    const long long m = q == 0 ? (pc[r] & kM20) : pc[r];
+    if (q >= 0 && m != 0)
+      atomicAdd(reinterpret_cast<unsigned long long*>(zd_col + q * stride), (unsigned long long)sgnd(m, P.sgn));
   }
 }
 
+// carry-normalise (value-preserving): digits 1..6 in [0, 2^30), digit 0 signed
+__device__ __forceinline__ void eda_normalize(long long (&D)[kL]) {
+#pragma unroll
+  for (int q = kL - 1; q >= 1; --q) {
+    const long long c = D[q] >> kW;  // arithmetic shift = floor division
+    D[q] -= c * (1ll << kW);
+    D[q - 1] += c;
+  }
+}
+
+// round(D) of the spec: the exact value's carry-normalised 40-bit digits N_0..N_4 (bits [-8, ..), [-48, -8), ...,
+// [-168, -128)), then v = 0; v = v + N_d * 2^B_d for d = 0..4, every conversion and addition rounded
 __device__ __forceinline__ double eda_round_d(const long long* Din) {
   long long D[kL];
 #pragma unroll
   for (int q = 0; q < kL; ++q) D[q] = Din[q];
-#pragma unroll
-  for (int q = kL - 1; q >= 1; --q) {
-    const long long c = D[q] >> 40;  // arithmetic shift = floor division
-    D[q] -= c * (1ll << 40);
-    D[q - 1] += c;
-  }
-  const double pw[kL] = {0x1p-8, 0x1p-48, 0x1p-88, 0x1p-128, 0x1p-168};
+  eda_normalize(D);
+  // D_q (q >= 1) covers bits [30 (6 - q), 30 (7 - q)) above 2^-168; D_0 sits at bit 180
+  const long long N4 = D[6] | ((D[5] & 0x3ff) << 30);
+  const long long N3 = (D[5] >> 10) | ((D[4] & 0xfffff) << 20);
+  const long long N2 = (D[4] >> 20) | (D[3] << 10);
+  const long long N1 = D[2] | ((D[1] & 0x3ff) << 30);
+  const long long N0 = (D[1] >> 10) + D[0] * (1ll << 20);
+  const long long N[5] = {N0, N1, N2, N3, N4};
+  const double pw[5] = {0x1p-8, 0x1p-48, 0x1p-88, 0x1p-128, 0x1p-168};
   double v = 0.0;
 #pragma unroll
-  for (int q = 0; q < kL; ++q) v = __dadd_rn(v, __dmul_rn(__ll2double_rn(D[q]), pw[q]));
+  for (int q = 0; q < 5; ++q) v = __dadd_rn(v, __dmul_rn(__ll2double_rn(N[q]), pw[q]));
   return v;
 }
 
@@ -545,24 +573,36 @@ __global__ void k_r_scalar_b(DevState* __restrict__ st, long long* __restrict__ 
 }
 
 // int64 digits <-> pairs of exact doubles (signed high 32 bits, unsigned low 32 bits) for the FP64 SUM allreduce:
-// every partial sum of P such halves is an integer below 2^53 in magnitude, hence exact in any order.
-__global__ void k_r_pack(const long long* __restrict__ src, int64_t n, int nseg, int64_t stride,
-                         double* __restrict__ buf) {
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n * nseg; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t sg = i / n, o = i - sg * n;
-    const long long v = src[sg * stride + o];
-    buf[2 * i] = (double)(v >> 32);
-    buf[2 * i + 1] = (double)(v & 0xffffffffll);
+// every partial sum of P such halves is an integer below 2^53 in magnitude, hence exact in any order.  nval values of
+// kL digits: digit q of value i at src[q * plane + i] (digit-major planes) or, plane == 0, at src[i * kL + q].  Each
+// value is carry-normalised first (value-preserving), so the rank sum of a digit stays below P * 2^30 whatever the
+// number of terms behind it.
+__device__ __forceinline__ int64_t dig_at(int64_t i, int q, int64_t plane) { return plane ? q * plane + i : i * kL + q; }
+
+__global__ void k_r_pack(const long long* __restrict__ src, int64_t nval, int64_t plane, double* __restrict__ buf) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nval; i += (int64_t)gridDim.x * blockDim.x) {
+    long long D[kL];
+#pragma unroll
+    for (int q = 0; q < kL; ++q) D[q] = src[dig_at(i, q, plane)];
+    eda_normalize(D);
+#pragma unroll
+    for (int q = 0; q < kL; ++q) {
+      const int64_t o = (int64_t)q * nval + i;
+      buf[2 * o] = (double)(D[q] >> 32);
+      buf[2 * o + 1] = (double)(D[q] & 0xffffffffll);
+    }
   }
 }
 
-__global__ void k_r_unpack(const double* __restrict__ buf, int64_t n, int nseg, int64_t stride,
-                           long long* __restrict__ dst) {
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n * nseg; i += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t sg = i / n, o = i - sg * n;
-    const unsigned long long hi = (unsigned long long)(long long)buf[2 * i];
-    const unsigned long long lo = (unsigned long long)(long long)buf[2 * i + 1];
-    dst[sg * stride + o] = (long long)((hi << 32) + lo);  // two's-complement wrap-around = the int64 sum
+__global__ void k_r_unpack(const double* __restrict__ buf, int64_t nval, int64_t plane, long long* __restrict__ dst) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nval; i += (int64_t)gridDim.x * blockDim.x) {
+#pragma unroll
+    for (int q = 0; q < kL; ++q) {
+      const int64_t o = (int64_t)q * nval + i;
+      const unsigned long long hi = (unsigned long long)(long long)buf[2 * o];
+      const unsigned long long lo = (unsigned long long)(long long)buf[2 * o + 1];
+      dst[dig_at(i, q, plane)] = (long long)((hi << 32) + lo);  // two's-complement wrap-around = the int64 sum
+    }
   }
 }
 
@@ -596,6 +636,7 @@ struct SdView {  // layout of the scalar digit buffer (see lsqr_internal.cuh)
 }  // namespace
 
 int64_t repro_digits_per_value() { return kL; }
+int64_t repro_max_terms() { return (int64_t)1 << 33; }
 int64_t repro_sd_size(int64_t n_constr) { return kL * (5 + n_constr); }
 long long* repro_sd_part(long long* sd, int64_t n_constr, int part) {
   const SdView V(sd, n_constr);
@@ -630,11 +671,10 @@ cudaError_t repro_step(int step, const ReproArgs& a, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-cudaError_t repro_pack(const long long* src, int64_t n, int nseg, int64_t stride, double* buf, int unpack,
-                       cudaStream_t s) {
-  if (n * nseg == 0) return cudaSuccess;
-  if (unpack) k_r_unpack<<<grid_for(n * nseg), kRedThreads, 0, s>>>(buf, n, nseg, stride, const_cast<long long*>(src));
-  else k_r_pack<<<grid_for(n * nseg), kRedThreads, 0, s>>>(src, n, nseg, stride, buf);
+cudaError_t repro_pack(const long long* src, int64_t nval, int64_t plane, double* buf, int unpack, cudaStream_t s) {
+  if (nval == 0) return cudaSuccess;
+  if (unpack) k_r_unpack<<<grid_for(nval), kRedThreads, 0, s>>>(buf, nval, plane, const_cast<long long*>(src));
+  else k_r_pack<<<grid_for(nval), kRedThreads, 0, s>>>(src, nval, plane, buf);
   return cudaGetLastError();
 }
 

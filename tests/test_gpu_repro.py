@@ -173,3 +173,25 @@ def test_repro_edge_cases_bitwise(avu, case):
     assert same(out["se"], ro["se"])
     for k in ("r1norm", "r2norm", "anorm", "acond", "arnorm", "xnorm"):
         assert same(out[k], ro[k]), k
+
+
+def test_repro_many_rows_no_overflow(avu):
+    """12 M rows: beta^2 and the global column each sum 12 M terms, more than the 2^23 the round-1 int64 digits held
+    (they wrapped silently on both sides).  x, se after 3 iterations bit-identical to the oracle's repro mode, and
+    within 1e-9 of the default mode's x (3 iterations: before any divergence onset of the two roundings)."""
+    w = W.C2.replace(n_stars=120_000, n_obs=12_000_000, seed=9)
+    kw = dict(itn_limit=3, atol=0, btol=0, conlim=0, fixed_count=True)
+    s = repro_solver(avu, w)
+    out = s.solve(**kw)
+    s.close()
+    S = oracle.System(w)
+    ro = oracle.solve_system(S, repro=True, **kw)
+    assert same(out["x"], ro["x"]), first_diff(out["x"], ro["x"])
+    assert same(out["se"], ro["se"])
+    assert out["bnorm"] == ro["bnorm"]
+    s = avu.Solver.synthetic(w)
+    s.precondition()
+    d = s.solve(**kw)
+    s.close()
+    assert abs(d["bnorm"] - out["bnorm"]) <= 1e-13 * out["bnorm"]
+    assert np.linalg.norm(d["x"] - out["x"]) <= 1e-9 * np.linalg.norm(out["x"])

@@ -49,6 +49,25 @@ def test_eda_special_values():
     assert oracle.eda_sum([0.1] * 10) == float(Fraction(0.1) * 10)
 
 
+def test_eda_many_terms_no_overflow():
+    """2^25 terms (more than the 2^23 a 64-bit digit holds): the sums the mode takes at C3 and above -- beta^2 over
+    all rows, the global column, alpha^2 over the astro columns -- stay exact.  Pinned to math.fsum (the correctly
+    rounded exact sum) and to closed forms; the round-1 int64 digits failed both (off by 2^16 at 2*10^7 terms)."""
+    import math
+    n = 1 << 25
+    rng = np.random.default_rng(7)
+    a = rng.uniform(0.5, 1.0, n)                  # all positive: every piece adds up in the same digits
+    s = oracle.eda_sum(a)
+    f = math.fsum(a)
+    assert abs(s - f) <= 2 * math.ulp(f), (s, f)  # exact sum + the documented final rounding chain
+    assert oracle.eda_sum(np.full(n, 0.75)) == 0.75 * n                      # exact closed form
+    assert oracle.eda_sum(np.full(n, 1.0 + 2.0**-52)) == n * (1.0 + 2.0**-52)  # low digits saturated too
+    b = a * a
+    b[1::2] *= -1.0                               # mixed signs, squares as in ||u||^2 partial pieces
+    s2, f2 = oracle.eda_sum(b), math.fsum(b)
+    assert abs(s2 - f2) <= 2 * math.ulp(abs(f2)) + 1e-300, (s2, f2)
+
+
 def permuted(S, rng):
     """Same system, rows in a random order, constraint entries reversed (every sum in a different order)."""
     P = copy.copy(S)
