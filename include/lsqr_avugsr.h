@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define LSQR_ABI_VERSION 1
+#define LSQR_ABI_VERSION 2
 #define LSQR_SLOTS 24
 
 typedef struct lsqr_ctx* lsqr_t;
@@ -113,9 +113,10 @@ typedef struct {
                               P:L1763-1767); the first nonzero istop is reported in istop_first */
   int32_t use_graph;       /* 1: replay the iteration as a CUDA graph (default for small systems) */
   int32_t poll_every;      /* host polls the stop flag every k iterations (<= 0 => 16) */
-  int32_t fused;           /* 0: two-pass iteration (aprod1 then aprod2; default).  1: fused single pass
-                              (SURVEY §8(f) NEXT-1): u_hat = A v - (alpha/beta) u_hat and z = A^T u_hat in ONE read
-                              of A, then v' = z/beta - beta v; same results up to rounding */
+  int32_t two_pass;        /* 0 (default, the zero-initialised struct): fused single pass:
+                              u_hat = A v - (alpha/beta) u_hat and z = A^T u_hat in ONE read of A, then
+                              v' = z/beta - beta v.  1: two-pass iteration (the paper's structure: aprod1, then
+                              aprod2, A read twice).  Same results up to rounding (ABI v2; v1 had `fused`, default 0) */
 } lsqr_solve_params;
 
 typedef struct {
@@ -196,7 +197,7 @@ int lsqr_get_precond(lsqr_t h, double* D);
  * of squares, the row dots of aprod1, the column sums of aprod2, ||u||, ||v|| and ddnorm -- as an exact,
  * order-independent digit accumulation rounded once, and every other step as one IEEE operation without FMA
  * contraction, in the order of Paige & Saunders' recurrence.  The iterates are then bit-identical run
- * to run and to the CPU oracle's repro mode, independent of scheduling; lsqr_solve_params.fused is ignored and the
+ * to run and to the CPU oracle's repro mode, independent of scheduling; lsqr_solve_params.two_pass is ignored and the
  * iteration is several times slower than the default path (verification mode).  With nranks > 1 the digits are
  * allreduced exactly (as pairs of exact doubles), so D, x, se and every scalar are bit-identical for ANY number of
  * ranks and any shard map.  Allocates 56 B per local column of digit storage (+ 112 B per shared column when

@@ -18,8 +18,8 @@
  *   orc_hash/orc_pm1 ............ splitmix64 published test vectors; exactness/range properties
  *   orc_star_counts/orc_shard ... brute force invariants (sum, bounds, pair symmetry; cover/disjoint/lower_bound)
  *   orc_generate* ............... structural invariants + golden FNV-1a checksums (tests/golden/, written by
- *                                 tests/golden/make_golden.py which calls only this oracle) + independent numpy
- *                                 re-implementation of the hash on small cases
+ *                                 tests/golden/make_golden.py which calls only this oracle) + an independent
+ *                                 pure-Python splitmix64/H and sampled fields regenerated from it
  *   orc_aprod1/orc_aprod2 ........ dense materialisation A@x, A.T@y (numpy); adjoint identity
  *   orc_colnorms/orc_scale ....... unit column norms of the scaled matrix; scaled solve == unscaled lstsq
  *   orc_lsqr ..................... numpy.linalg.lstsq/QR; scipy.sparse.linalg.lsqr iterates; reorthogonalised mode

@@ -268,9 +268,9 @@ class Solver:
     # ------------------------------------------------------------------ LSQR
     @staticmethod
     def _params(itn_limit=100, atol=1e-8, btol=1e-8, conlim=1e8, damp=0.0, fixed_count=False, use_graph=True,
-                poll_every=16, fused=False):
+                poll_every=16, fused=True):
         return _capi.SolveParams(int(itn_limit), atol, btol, conlim, damp, int(bool(fixed_count)),
-                                 int(bool(use_graph)), int(poll_every), int(bool(fused)))
+                                 int(bool(use_graph)), int(poll_every), int(not fused))
 
     def solve(self, x_out=None, se_out=None, **kw):
         """Full solve; returns dict(result fields, x, se) with x, se as numpy (host) unless device tensors are

@@ -42,7 +42,7 @@ class GenParams(C.Structure):
 
 class SolveParams(C.Structure):
     _fields_ = [("itn_limit", i64), ("atol", d), ("btol", d), ("conlim", d), ("damp", d), ("fixed_count", i32),
-                ("use_graph", i32), ("poll_every", i32), ("fused", i32)]
+                ("use_graph", i32), ("poll_every", i32), ("two_pass", i32)]
 
 
 class Result(C.Structure):
@@ -94,12 +94,9 @@ def lib(build_if_missing: bool = True):
     global _lib
     with _lock:
         if _lib is None:
-            if build_if_missing:
-                try:
-                    _build.build()
-                except Exception:
-                    if not os.path.exists(_build.LIB):
-                        raise
+            if build_if_missing and _build.needs_build():
+                # sources newer than the library (or no library): a failed build must not silently load a stale .so
+                _build.build()
             if not os.path.exists(_build.LIB):
                 raise RuntimeError(f"CUDA extension {_build.LIB} is missing (run __graft_entry__.build())")
             L = C.CDLL(_build.LIB, mode=C.RTLD_GLOBAL)

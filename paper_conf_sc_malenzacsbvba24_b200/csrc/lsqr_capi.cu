@@ -111,6 +111,8 @@ struct lsqr_ctx {
   std::vector<double> cval_raw;
   // state
   bool poisoned = false, have_system = false, b_valid = false, preconditioned = false, initialized = false;
+  int64_t n_enq = 0;        // iterations enqueued since lsqr_init (lsqr_iterate's stop-flag bookkeeping)
+  int64_t itn_at_init = 0;  // device itn after lsqr_init (0; lsqr_set_state may change it)
   lsqr_solve_params params{};
   cudaGraphExec_t gexec = nullptr;
   bool graph_ok = false;
@@ -284,16 +286,16 @@ int enqueue_repro(lsqr_t h, int init) {
 
 // ------------------------------------------------------------------------------------------------ iteration
 // One LSQR iteration, all stream-ordered on h->s.  timing: optional events around the two
-// products ([0..1] aprod1, [2..3] aprod2).
+// products ([0..1] aprod1 or the fused row pass, [2..3] aprod2 or the column pass after the fused row pass).
+// Both variants leave the same state after their row pass(es) -- z = A^T u_hat with the UNNORMALISED u_hat in zA
+// (astro) and z_sh (shared slice) -- and finish with the same kernels (v' = z / beta - beta v, scalars, column update):
+//   fused (NEXT-1, default): k_fused3<R3_FUSED> reads A once (u_hat update and A^T u_hat in one pass);
+//   two-pass (the paper's structure): k_aprod1, then k_fused3<R3_AP2> (aprod2 on the fused kernel's loop).
 int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   SysView& S = h->S;
   cudaStream_t s = h->s;
   const bool multi = h->multi;
-  const bool fused = h->params.fused != 0;
-  // two-pass: k_aprod1, then aprod2 on the fused kernel's loop (k_fused3<R3_AP2>); afterwards the state is the
-  // fused pass's (unnormalised z in zA / z_sh), finished by the same kernels
-  const bool lean2 = !fused && lean_products_ok(S);
-  const bool fstate = fused || lean2;
+  const bool fused = h->params.two_pass == 0;
   if (h->repro) {  // NEXT-4: 7 launches (+ 4 x pack/unpack when P > 1), all in lsqr_repro.cu
     if (ev) cudaEventRecord(ev[0], s);
     CKR(enqueue_repro(h, 0));
@@ -301,61 +303,43 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
     return LSQR_OK;
   }
   if (ev) cudaEventRecord(ev[0], s);
-  if (fused) {  // NEXT-1: u_hat update and A^T u_hat in one read of A
+  if (fused) {
     CKL(h, launch_fused(S, h->grid, h->v, h->u, h->zA, h->zsh, h->part_rows, h->cpart, h->st, s), "fused");
   } else {
     CKL(h, launch_aprod1(AP1_LSQR, S, h->grid, h->v, h->u, h->part_rows, h->cpart, h->st, s), "aprod1");
   }
   if (ev) cudaEventRecord(ev[1], s);
-  if (lean2) {  // z = A^T u_hat with the unnormalised u_hat (beta is applied afterwards, as in the fused pass)
+  if (!fused) {
     if (ev) cudaEventRecord(ev[2], s);
     CKL(h, launch_ap2_lean(S, h->grid, h->u, h->zA, h->zsh, h->st, s), "aprod2");
     if (ev) cudaEventRecord(ev[3], s);
   }
-  if (fstate && !multi) {  // fused: 4 launches (rows, post = beta + v' everywhere, scalar, column update); lean2: 5
-    if (ev && !lean2) cudaEventRecord(ev[2], s);
-    CKL(h, launch_post(S, h->v, h->zA, h->zsh, h->part_rows, fused ? h->grid : h->W, h->cpart, h->uc, h->uc_tmp,
-                       h->part_va, kG3, h->st, s), "post");
-    if (ev && !lean2) cudaEventRecord(ev[3], s);
+  const int64_t n_b2 = fused ? h->grid : h->W;  // k_fused3 publishes one beta^2 partial per CTA, k_aprod1 per warp
+  if (!multi) {  // fused: 4 launches (rows, post = beta + v' everywhere, scalar, column update); two-pass: 5
+    if (ev && fused) cudaEventRecord(ev[2], s);
+    CKL(h, launch_post(S, h->v, h->zA, h->zsh, h->part_rows, n_b2, h->cpart, h->uc, h->uc_tmp, h->part_va, kG3,
+                       h->st, s), "post");
+    if (ev && fused) cudaEventRecord(ev[3], s);
     CKL(h, launch_scalar(h->st, h->part_va, kG3, nullptr, 0, h->part_wa, kG3, h->part_ws, kG3, nullptr, nullptr, 0,
                          h->hflag_dev, s, h->uc_tmp, h->uc, h->ucn, (int)h->n_constr), "scalar");
     CKL(h, launch_colupdate(h->v, h->w, h->x, h->var, h->n_loc_cols, S.A0, h->part_wa, h->part_ws, kG3, h->st, s),
         "colupdate");
     return LSQR_OK;
   }
-  const int64_t n_b2 = fused ? h->grid : h->W;  // k_fused3 publishes one beta^2 partial per CTA, k_aprod1 per warp
-  if (!multi) {
-    CKL(h, launch_beta(0, S, h->part_rows, n_b2, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta");
-  } else {
-    CKL(h, launch_beta(1, S, h->part_rows, n_b2, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta1");
-    // AR1 payload: [constraint dots | beta^2 local | ||w_astro||^2 local]
-    CKL(h, launch_sum_to(h->part_wa, kG3, h->ar1 + h->n_constr + 1, s), "wsum");
-    CKR(allreduce(h, h->ar1, h->n_constr + 2));
-    CKL(h, launch_beta(2, S, h->part_rows, n_b2, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta2");
-  }
-  if (ev && !lean2) cudaEventRecord(ev[2], s);
-  const double* a2part;
-  int64_t n_a2;
-  if (fstate) {
-    CKL(h, launch_vastro(S, h->v, h->zA, h->uc, h->zsh, h->part_va, kG3, h->st, h->rank == 0, s), "vastro");
-    a2part = h->part_va;
-    n_a2 = kG3;
-  } else {
-    CKL(h, launch_aprod2(AP2_LSQR, S, h->grid, h->u, h->ucn, h->v, h->zsh, h->part_a2, h->st, h->rank == 0, s),
-        "aprod2");
-    a2part = h->part_a2;
-    n_a2 = h->W;
-  }
-  if (ev && !lean2) cudaEventRecord(ev[3], s);
-  if (multi) {
-    // AR2 payload: [z_att | z_instr | z_glob | alpha^2 astro local]
-    CKL(h, launch_sum_to(a2part, n_a2, h->zsh + h->n_sh, s), "a2sum");
-    CKR(allreduce(h, h->zsh, h->n_sh + 1));
-  }
-  CKL(h, launch_vshared(S, h->v + S.A0, h->zsh, h->part_sh, kG2, h->st, fstate ? 1 : 0, s), "vshared");
-  CKL(h, launch_scalar(h->st, a2part, n_a2, h->part_sh, kG2, h->part_wa, kG3, h->part_ws, kG3,
-                       multi ? h->zsh + h->n_sh : nullptr, multi ? h->ar1 + h->n_constr + 1 : nullptr, 0,
-                       h->hflag_dev, s),
+  // P > 1: beta needs AR1 = [constraint dots | beta^2 local | ||w_astro||^2 local]
+  CKL(h, launch_beta(1, S, h->part_rows, n_b2, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta1");
+  CKL(h, launch_sum_to(h->part_wa, kG3, h->ar1 + h->n_constr + 1, s), "wsum");
+  CKR(allreduce(h, h->ar1, h->n_constr + 2));
+  CKL(h, launch_beta(2, S, h->part_rows, n_b2, h->cpart, h->ar1, h->uc, h->ucn, h->crhs, h->st, 0, s), "beta2");
+  if (ev && fused) cudaEventRecord(ev[2], s);
+  CKL(h, launch_vastro(S, h->v, h->zA, h->uc, h->zsh, h->part_va, kG3, h->st, h->rank == 0, s), "vastro");
+  if (ev && fused) cudaEventRecord(ev[3], s);
+  // AR2 payload: [z_att | z_instr | z_glob | alpha^2 astro local]
+  CKL(h, launch_sum_to(h->part_va, kG3, h->zsh + h->n_sh, s), "a2sum");
+  CKR(allreduce(h, h->zsh, h->n_sh + 1));
+  CKL(h, launch_vshared(S, h->v + S.A0, h->zsh, h->part_sh, kG2, h->st, 1, s), "vshared");
+  CKL(h, launch_scalar(h->st, h->part_va, kG3, h->part_sh, kG2, h->part_wa, kG3, h->part_ws, kG3, h->zsh + h->n_sh,
+                       h->ar1 + h->n_constr + 1, 0, h->hflag_dev, s),
       "scalar");
   CKL(h, launch_colupdate(h->v, h->w, h->x, h->var, h->n_loc_cols, S.A0, h->part_wa, h->part_ws, kG3, h->st, s),
       "colupdate");
@@ -364,8 +348,8 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
 
 int kernels_per_iteration(lsqr_t h) {
   if (h->repro) return h->multi ? 15 : 7;
-  if (h->params.fused) return h->multi ? 9 : 4;
-  return lean_products_ok(h->S) ? (h->multi ? 10 : 5) : (h->multi ? 9 : 6);
+  if (!h->params.two_pass) return h->multi ? 9 : 4;
+  return h->multi ? 10 : 5;
 }
 
 int build_graph(lsqr_t h) {
@@ -997,6 +981,8 @@ int lsqr_init(lsqr_t h, const lsqr_solve_params* p) {
   if (!h->b_valid) return fail(h, LSQR_ESTATE, "b was consumed by a previous solve; regenerate or set_system");
   h->params = *p;
   if (h->params.poll_every <= 0) h->params.poll_every = 16;
+  h->n_enq = 0;
+  h->itn_at_init = 0;
   SysView& S = h->S;
   const bool multi = h->multi;
   enter(h);
@@ -1061,6 +1047,7 @@ int lsqr_iterate(lsqr_t h, int64_t n_iter) {
   CKC(h, cudaEventCreateWithFlags(&evs[0], cudaEventDisableTiming));
   CKC(h, cudaEventCreateWithFlags(&evs[1], cudaEventDisableTiming));
   int64_t done = 0, batch = 0;
+  int64_t enq_end[2] = {0, 0};  // iterations enqueued since lsqr_init at the end of batch b (slot b & 1)
   int rc = LSQR_OK;
   while (done < n_iter && rc == LSQR_OK) {
     const int64_t nb = std::min(k, n_iter - done);
@@ -1073,10 +1060,17 @@ int lsqr_iterate(lsqr_t h, int64_t n_iter) {
       }
     }
     done += nb;
+    h->n_enq += nb;
+    enq_end[batch & 1] = h->n_enq;
     cudaEventRecord(evs[batch & 1], h->s);
     if (batch > 0) {  // wait for the previous batch, then poll the stop flag (device-written, host-mapped)
       cudaEventSynchronize(evs[(batch - 1) & 1]);
-      if (*(volatile int32_t*)h->hflag & 1) break;
+      // The flag is written by every scalar step, so it may already come from batch b, still running.  Stop only on
+      // a halt that happened within the FINISHED batches (its iteration count <= the count enqueued by the end of
+      // batch b-1): the halting iteration is the same on every rank, so all ranks stop after the same batch and
+      // issue the same collectives (a halt seen early is acted on after the next batch).
+      const int32_t f = *(volatile int32_t*)h->hflag;
+      if ((f & 1) && (int64_t)(f >> 1) <= enq_end[(batch - 1) & 1] + h->itn_at_init) break;
     }
     ++batch;
   }
@@ -1165,7 +1159,7 @@ int lsqr_set_state(lsqr_t h, const double* sc, const double* u, const double* v,
   enter(h);
   CKC(h, cudaStreamSynchronize(h->s));
   DevState st;
-  CKC(h, cudaMemcpy(&st, h->st, sizeof st, cudaMemcpyDeviceToHost));
+  CKC(h, cudaMemcpy(&st, h->st, sizeof st, cudaMemcpyDeviceToHost));  // h->s is idle (synchronised above)
   if (sc) {
     st.alpha = sc[LSQR_S_ALPHA]; st.beta = sc[LSQR_S_BETA]; st.rhobar = sc[LSQR_S_RHOBAR];
     st.phibar = sc[LSQR_S_PHIBAR]; st.anorm = sc[LSQR_S_ANORM]; st.acond = sc[LSQR_S_ACOND];
@@ -1177,22 +1171,23 @@ int lsqr_set_state(lsqr_t h, const double* sc, const double* u, const double* v,
     st.halted = (int32_t)sc[LSQR_S_HALTED];
   }
   if (u) {  // the given u is normalised: store it as u_hat with inv_beta = 1
-    CKC(h, cudaMemcpy(h->u, u, sizeof(double) * h->n_loc_rows, cudaMemcpyHostToDevice));
+    CKC(h, cudaMemcpyAsync(h->u, u, sizeof(double) * h->n_loc_rows, cudaMemcpyHostToDevice, h->s));
     if (h->n_constr) {
-      CKC(h, cudaMemcpy(h->uc, u + h->n_loc_rows, sizeof(double) * h->n_constr, cudaMemcpyHostToDevice));
-      CKC(h, cudaMemcpy(h->ucn, u + h->n_loc_rows, sizeof(double) * h->n_constr, cudaMemcpyHostToDevice));
+      CKC(h, cudaMemcpyAsync(h->uc, u + h->n_loc_rows, sizeof(double) * h->n_constr, cudaMemcpyHostToDevice, h->s));
+      CKC(h, cudaMemcpyAsync(h->ucn, u + h->n_loc_rows, sizeof(double) * h->n_constr, cudaMemcpyHostToDevice, h->s));
     }
     st.inv_beta = 1.0;
   }
+  h->itn_at_init = (int64_t)st.itn - h->n_enq;  // lsqr_iterate: device itn = itn_at_init + iterations enqueued
   st.u_scale = st.alpha * st.inv_beta;
   st.v_pending = 0;
   st.col_enable = 0;
-  CKC(h, cudaMemcpy(h->st, &st, sizeof st, cudaMemcpyHostToDevice));
+  CKC(h, cudaMemcpyAsync(h->st, &st, sizeof st, cudaMemcpyHostToDevice, h->s));
   const size_t nb = sizeof(double) * h->n_loc_cols;
-  if (v) CKC(h, cudaMemcpy(h->v, v, nb, cudaMemcpyHostToDevice));
-  if (w) CKC(h, cudaMemcpy(h->w, w, nb, cudaMemcpyHostToDevice));
-  if (x) CKC(h, cudaMemcpy(h->x, x, nb, cudaMemcpyHostToDevice));
-  if (var) CKC(h, cudaMemcpy(h->var, var, nb, cudaMemcpyHostToDevice));
+  if (v) CKC(h, cudaMemcpyAsync(h->v, v, nb, cudaMemcpyHostToDevice, h->s));
+  if (w) CKC(h, cudaMemcpyAsync(h->w, w, nb, cudaMemcpyHostToDevice, h->s));
+  if (x) CKC(h, cudaMemcpyAsync(h->x, x, nb, cudaMemcpyHostToDevice, h->s));
+  if (var) CKC(h, cudaMemcpyAsync(h->var, var, nb, cudaMemcpyHostToDevice, h->s));
   // ||w||^2 partials (astro / shared) for the next iteration's ddnorm
   CKL(h, launch_sumsq(h->w, h->S.A0, h->part_wa, kG3, h->s), "wsum_a");
   CKL(h, launch_sumsq(h->w + h->S.A0, h->n_sh, h->part_ws, kG3, h->s), "wsum_s");
@@ -1250,11 +1245,12 @@ int lsqr_solve(lsqr_t h, const lsqr_solve_params* p, lsqr_result* res, double* x
     res->t_iter_max_over_ranks_s = res->t_iter_mean_s;
     if (h->multi && h->comm_kind == LSQR_COMM_NCCL) {
       double t = res->t_iter_mean_s;
-      CKC(h, cudaMemcpy(h->tmax, &t, sizeof t, cudaMemcpyHostToDevice));
+      CKC(h, cudaMemcpyAsync(h->tmax, &t, sizeof t, cudaMemcpyHostToDevice, h->s));
       ncclResult_t r = g_nccl.AllReduce(h->tmax, h->tmax, 1, ncclFloat64, ncclMax, h->nccl, h->s);
       if (r != ncclSuccess) return fail(h, LSQR_ENCCL, "ncclAllReduce(max)");
       CKC(h, cudaStreamSynchronize(h->s));
-      CKC(h, cudaMemcpy(&t, h->tmax, sizeof t, cudaMemcpyDeviceToHost));
+      CKC(h, cudaMemcpyAsync(&t, h->tmax, sizeof t, cudaMemcpyDeviceToHost, h->s));
+      CKC(h, cudaStreamSynchronize(h->s));
       res->t_iter_max_over_ranks_s = t;
     }
   }

@@ -156,12 +156,11 @@ cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* p
 // NEXT-1 fused single pass (u_hat update + A^T u_hat in one read of A) and its astro column pass
 cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh,
                          double* part, double* cpart, const DevState* st, cudaStream_t s);
-// the two-pass iteration's aprod2 on the fused kernel's loop (k_fused3<R3_AP2>): z = A^T u_hat (unnormalised) into
-// zA / z_sh, the state the fused pass leaves; needs the instrumental slice in shared memory (lean_products_ok)
-bool lean_products_ok(const SysView& S);
 // lsqr_aprod2 after k_fused3<R3_AP2>: x_astro += zA + astro constraint entries . y_c; shared constraint entries -> z_sh
 cudaError_t launch_astro_add(const SysView& S, double* x, const double* zA, const double* yc, double* zsh,
                              int do_shared_constr, cudaStream_t s);
+// the two-pass iteration's aprod2 on the fused kernel's loop (k_fused3<R3_AP2>): z = A^T u_hat (unnormalised) into
+// zA / z_sh, the state the fused pass leaves (every instrumental-slice size: the IG regime covers large ones)
 cudaError_t launch_ap2_lean(const SysView& S, int grid, const double* u, double* zA, double* zsh, const DevState* st,
                             cudaStream_t s);
 cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const double* uc, double* zsh, double* part,

@@ -8,7 +8,10 @@
 // which makes the attitude gathers (aprod1) and REDs (aprod2) sector-coalesced.
 #include <algorithm>
 #include <cstdlib>
+#include <map>
+#include <mutex>
 #include <type_traits>
+#include <utility>
 
 #include "lsqr_internal.cuh"
 
@@ -1542,17 +1545,28 @@ cudaError_t launch_generate(const GenArgs& g, double* vals, IdxRec* idx, const i
   return cudaGetLastError();
 }
 
+// Dynamic shared-memory opt-in of a kernel, per (kernel, device): the attribute applies to the device current at
+// the call, and handles of one process may live on different devices or threads.
+static cudaError_t ensure_smem(const void* fn, size_t bytes) {
+  static std::mutex mu;
+  static std::map<std::pair<const void*, int>, size_t> done;
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  std::lock_guard<std::mutex> g(mu);
+  size_t& cur = done[{fn, dev}];
+  if (bytes <= cur) return cudaSuccess;
+  e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  if (e == cudaSuccess) cur = bytes;
+  return e;
+}
+
 template <int MODE, bool SM>
 static cudaError_t ap1(const SysView& S, int grid, const double* x, double* y, double* part, double* cpart,
                        const DevState* st, cudaStream_t s) {
   const size_t smem = kRingBytes + kBarBytes + (SM ? (size_t)S.ip.slots() * sizeof(double) : 0);
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_aprod1<MODE, SM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)(kRingBytes + kBarBytes + (SM ? (kInstrSmemMax + 64) * sizeof(double) : 0)));
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
+  cudaError_t e = ensure_smem((const void*)k_aprod1<MODE, SM>, smem);
+  if (e != cudaSuccess) return e;
   k_aprod1<MODE, SM><<<grid, kThreads, smem, s>>>(S, x, y, part, cpart, st);
   return cudaGetLastError();
 }
@@ -1570,13 +1584,8 @@ template <int MODE, bool SM>
 static cudaError_t ap2(const SysView& S, int grid, const double* y, const double* ucn, double* xv, double* zsh,
                        double* part, const DevState* st, int dsc, cudaStream_t s) {
   size_t smem = kRingBytes + kBarBytes + (SM ? (size_t)S.ip.slots() * sizeof(double) : 0);
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_aprod2<MODE, SM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)(kRingBytes + kBarBytes + (SM ? (kInstrSmemMax + 64) * sizeof(double) : 0)));
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
+  cudaError_t e = ensure_smem((const void*)k_aprod2<MODE, SM>, smem);
+  if (e != cudaSuccess) return e;
   k_aprod2<MODE, SM><<<grid, kThreads, smem, s>>>(S, y, ucn, xv, zsh, part, st, dsc);
   return cudaGetLastError();
 }
@@ -1648,13 +1657,8 @@ static F3Plan f3_plan(const SysView& S) {
 template <int KIND, int DIAG, bool SMATT, bool IG, bool ZREP>
 static cudaError_t fz3v(const SysView& S, const F3Plan& P, int grid, const double* x, double* u, double* zA,
                         double* zsh, double* part, double* cpart, const DevState* st, cudaStream_t s) {
-  static size_t attr_set = 0;
-  if (P.smem > attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(k_fused3<KIND, DIAG, SMATT, IG, ZREP>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)P.smem);
-    if (e != cudaSuccess) return e;
-    attr_set = P.smem;
-  }
+  cudaError_t e = ensure_smem((const void*)k_fused3<KIND, DIAG, SMATT, IG, ZREP>, P.smem);
+  if (e != cudaSuccess) return e;
   SysView S2 = S;
   S2.f3_zrep = P.zrep;
   S2.f3_arep = P.arep;
@@ -1705,7 +1709,6 @@ cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u,
   return fz3<R3_FUSED, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
 }
 
-bool lean_products_ok(const SysView&) { return true; }  // k_fused3 covers every instrumental-slice size (IG)
 cudaError_t launch_ap2_lean(const SysView& S, int grid, const double* u, double* zA, double* zsh, const DevState* st,
                             cudaStream_t s) {
   return fz3<R3_AP2, 0>(S, grid, nullptr, const_cast<double*>(u), zA, zsh, nullptr, nullptr, st, s);

@@ -34,7 +34,7 @@ def test_library_exports_every_declared_symbol():
     for n in names:
         assert hasattr(L, n), n
     assert set(names) == set(_capi.EXPORTS), set(names) ^ set(_capi.EXPORTS)
-    assert L.lsqr_abi_version() == 1
+    assert L.lsqr_abi_version() == 2
     assert L.lsqr_strerror(-6) == b"rows not grouped by star / inconsistent with obs_per_star"
 
 

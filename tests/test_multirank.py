@@ -113,6 +113,15 @@ def _gpu_worker(rank, world, port, q, itn, fused):
         s.precondition()
         D = s.get_precond()
         out = s.solve(itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True, use_graph=False, fused=fused)
+        # early convergence (fixed_count off): every rank must stop after the same iteration (lsqr_iterate's stop
+        # decision may only depend on finished batches, else ranks issue different collectives)
+        s.generate(w.seed)
+        s.precondition()
+        early = s.solve(itn_limit=500, atol=1e-9, btol=1e-9, fused=fused, poll_every=3)
+        dist_obj = __import__("torch.distributed", fromlist=["all_gather_object"])
+        its = [None] * world
+        dist_obj.all_gather_object(its, (early["itn"], early["istop"]))
+        assert len(set(its)) == 1, its
         # plain products through the ABI
         xg = torch.ones(s.n_local_cols, dtype=torch.float64, device="cuda")
         yg = torch.zeros(s.n_local_rows + s.n_constr, dtype=torch.float64, device="cuda")
@@ -279,3 +288,24 @@ def test_gpu_nccl_path_forced_on_one_rank(cuda_device, mode):
         assert rel(b["x"], a["x"]) <= 1e-9 and abs(b["r1norm"] - a["r1norm"]) <= 1e-10 * a["r1norm"]
     assert np.allclose(prods[0][0], prods[1][0], rtol=1e-12, atol=1e-12)
     assert np.allclose(prods[0][1], prods[1][1], rtol=1e-12, atol=1e-12)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("fused", [False, True], ids=["twopass", "fused"])
+def test_gpu_nccl_forced_early_stop(cuda_device, fused):
+    """Early convergence through the asynchronous NCCL path (graph-captured collectives, stop flag polled every 3
+    iterations while the next batch runs): the stop is taken after the batch in which the halting iteration ran,
+    so itn, istop and x equal the single-rank path's (a decision based on a flag written by a batch still
+    in flight could make ranks disagree on the number of batches)."""
+    import paper_conf_sc_malenzacsbvba24_b200 as avu
+    w = W.C1C.replace(jitter_pct=50)
+    outs = []
+    for force in (False, True):
+        s = avu.Solver.synthetic(w, force_collectives=force)
+        s.precondition()
+        outs.append(s.solve(itn_limit=500, atol=1e-9, btol=1e-9, fused=fused, poll_every=3, use_graph=True))
+        s.close()
+    a, b = outs
+    assert 0 < a["itn"] < 500 and a["istop"] in (1, 2)
+    assert a["istop"] == b["istop"] and abs(a["itn"] - b["itn"]) <= 2  # SURVEY 8(c): |d itn| <= 2 across roundings
+    assert np.linalg.norm(a["x"] - b["x"]) <= 1e-8 * np.linalg.norm(a["x"])

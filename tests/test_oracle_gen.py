@@ -33,11 +33,41 @@ def test_splitmix64_reference_vectors():
     assert got == ref
 
 
+def _py_mix(z):
+    """splitmix64 finaliser in plain Python integers (mod 2^64), written from the published algorithm."""
+    M = 2**64
+    z = (z + 0x9E3779B97F4A7C15) % M
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) % M
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) % M
+    return z ^ (z >> 31)
+
+
+def _py_hash(seed, tag, i, j):
+    return _py_mix(_py_mix(_py_mix(seed ^ ((tag << 56) % 2**64)) ^ i) ^ j)
+
+
 def test_hash_composition():
-    L = oracle.lib()
-    for seed, tag, i, j in [(1, 4, 0, 0), (20241117, 2, 123456789, 0), (7, 8, 5, 99)]:
-        h = L.orc_mix(L.orc_mix(L.orc_mix(seed ^ (tag << 56)) ^ i) ^ j)
-        assert oracle.hash64(seed, tag, i, j) == h
+    """H(seed, tag, i, j) of O-GEN against an independent pure-Python implementation (not the oracle's orc_mix)."""
+    for seed, tag, i, j in [(1, 4, 0, 0), (20241117, 2, 123456789, 0), (7, 8, 5, 99), (2**64 - 1, 255, 2**40, 23)]:
+        assert oracle.hash64(seed, tag, i, j) == _py_hash(seed, tag, i, j)
+
+
+def test_generated_fields_match_independent_hash():
+    """A sample of generated entries (values, attitude k0, instrumental columns, hashed b) recomputed from the
+    O-GEN spec with the pure-Python hash above: the oracle's generator applies the spec (docs/GENERATOR.md)."""
+    w = W.C1.replace(jitter_pct=50, seed=29)
+    S = oracle.System(w)
+    n_axis, g = w.n_att // 3, w.n_instr // 6
+    A0, I0 = 5 * w.n_stars, 5 * w.n_stars + w.n_att
+    pm1 = lambda h: ((h >> 10) - 2**53) / 2.0**53
+    for i in [0, 1, 17, 999, 12345, w.n_obs - 1]:
+        for s_ in (0, 4, 5, 16, 17, 22, 23):
+            assert S.vals[i, s_] == pm1(_py_hash(w.seed, 4, i, s_))
+        k0 = _py_hash(w.seed, 2, i, 0) % (n_axis - 3)
+        assert S.mT[i] == A0 + k0
+        for jj in range(6):
+            assert S.iC[i, jj] == I0 + jj * g + _py_hash(w.seed, 3, i, jj) % g
+        assert S.b[i] == pm1(_py_hash(w.seed, 5, i, 0))
 
 
 def test_pm1_exact_and_range():
