@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """Benchmark: seconds per LSQR iteration and HBM-roofline fraction (FP64) of the AVU-GSR hot path on B200.
 
-    python bench.py [--gpus N --steps K --warmup W --config C2]          # our CUDA path (one JSON line)
+    python bench.py [--gpus N --steps K --warmup W --config C3]          # our CUDA path (one JSON line)
     python bench.py --impl reference ...                                  # the CPU oracle (reference arm)
     torchrun --nproc-per-node N bench.py --gpus N ...                     # multi-GPU, weak scaling
 
@@ -120,23 +120,77 @@ def load_traffic(workload, kernel):
 
 
 # ------------------------------------------------------------------------------------------------ cpu baseline
-def cpu_baseline(w, iters=3, repro=False):
-    """The oracle (serial C, as it stands) on a bounded sample: the full system, `iters` LSQR iterations
-    (``repro``: the oracle's bitwise-reproducible mode, NEXT-4)."""
+def oracle_sample(w):
+    """A bounded sample of workload w for timing the CPU oracle: the rows of shard 0 of P (O-SHARD; P = 1 for systems
+    up to ~7 M rows), with w's full column dimension.  Returns (System, P)."""
+    import oracle
+    P = max(1, -(-w.n_obs // 7_000_000))
+    S = oracle.System(w, rank=0, nranks=P)
+    return S, P
+
+
+def _time_products(S, fns, reps=2):
+    """Median wall time of one aprod1 + one aprod2 call on the sample (the part of an iteration that scales with
+    the rows; the n-vector updates do not)."""
+    x = np.full(S.n_cols, 1e-3)
+    y = np.zeros(S.m_local)
+    ts = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        fns[0](x, y)
+        fns[1](y, x)
+        ts.append(time.perf_counter() - t0)
+    return float(np.median(ts))
+
+
+def cpu_baseline(w, iters=3, repro=False, all_cores=True):
+    """The oracle on a bounded sample of w (oracle_sample): `iters` timed fixed-count LSQR iterations of (a) the
+    serial C checker as it stands (one core) and (b) its all-core OpenMP timing build (oracle/omp_timing.c: the same
+    source with OpenMP loops and products; ``repro``: the serial repro mode only).  The sample covers 1/P of the rows
+    with the full column dimension, so the full-workload time per iteration is extrapolated as
+    t_iter(sample) + (P - 1) * t_products(sample) (the products scale with the rows, the n-vector updates do not)."""
+    import ctypes
     import oracle
     t0 = time.perf_counter()
-    S = oracle.System(w)
+    S, P = oracle_sample(w)
     S.apply_precond(repro=repro)
     t_setup = time.perf_counter() - t0
     stamps = []
     oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), atol=0, btol=0, conlim=0, itn_limit=iters + 1, fixed_count=True,
                 want_se=False, trace=lambda st: stamps.append(time.perf_counter()), trace_vectors=False, repro=repro)
     per = [b - a for a, b in zip(stamps[:-1], stamps[1:])]
-    v = float(np.median(per))
-    return {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"full {w.name} system ({w.n_obs} rows), {len(per)} timed LSQR iterations of the serial C "
-                      f"oracle{' (repro mode)' if repro else ''} after 1 untimed (setup {t_setup:.1f} s excluded)",
-            "cpu_model": _cpu_model(), "host_cores": os.cpu_count()}
+    t_it = float(np.median(per))
+    t_pr = _time_products(S, (S.aprod1_repro, S.aprod2_repro) if repro else (S.aprod1, S.aprod2)) if P > 1 else 0.0
+    serial = {"value": t_it + (P - 1) * t_pr, "cores": 1, "sample_s_per_iter": t_it, "sample_products_s": t_pr}
+    sample = (f"rows of shard 0 of {P} of {w.name} ({S.n_rows} of {w.n_obs} rows; all {S.n_cols} columns), "
+              f"{len(per)} timed LSQR iterations after 1 untimed; full-system s/iteration extrapolated as "
+              f"t_iter + (P-1) * t(aprod1 + aprod2) on the sample (setup {t_setup:.1f} s excluded)")
+    out = {"value": serial["value"], "unit": UNIT, "cores": 1, "kind": "oracle",
+           "sample": sample, "serial": serial, "cpu_model": _cpu_model(), "host_cores": os.cpu_count()}
+    if all_cores and not repro:
+        r = oracle.time_lsqr_omp(S, iters)
+        L = oracle.omp_lib()
+        fns = (lambda x, y: L.orc_omp_aprod1(ctypes.byref(S.S), oracle._p(x), oracle._p(y)),
+               lambda y, x: L.orc_omp_aprod2(ctypes.byref(S.S), oracle._p(y), oracle._p(x)))
+        o_it = float(np.median(r["per_iter_s"]))
+        o_pr = _time_products(S, fns) if P > 1 else 0.0
+        omp = {"value": o_it + (P - 1) * o_pr, "cores": r["threads"], "sample_s_per_iter": o_it,
+               "sample_products_s": o_pr,
+               "build": "oracle/omp_timing.c (the oracle source with OpenMP loops/products; timing only)"}
+        out.update(value=omp["value"], cores=omp["cores"], kind="oracle (all-core OpenMP timing build)",
+                   all_cores=omp)
+    return out
+
+
+def _mem_available():
+    """MemAvailable of this host in bytes (None if unknown)."""
+    try:
+        for line in open("/proc/meminfo"):
+            if line.startswith("MemAvailable:"):
+                return int(line.split()[1]) * 1024
+    except Exception:
+        pass
+    return None
 
 
 def _cpu_model():
@@ -211,30 +265,38 @@ def workload_of(args):
 
 # ------------------------------------------------------------------------------------------------ reference arm
 def run_reference(args):
+    """Reference arm: the CPU oracle (this tier has no reference implementation; the oracle is the base contract's
+    reference) timed on the host cores -- its all-core OpenMP timing build -- on the same config, each step one LSQR
+    iteration over the bounded sample of oracle_sample(), extrapolated to the full workload as in cpu_baseline()."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
-    base = workload_of(args)
-    w = base
+    w = workload_of(args)
+    import ctypes
     import oracle
     t0 = time.perf_counter()
-    S = oracle.System(w)
+    S, P = oracle_sample(w)
     S.apply_precond()
     setup = time.perf_counter() - t0
-    stamps = [time.perf_counter()]
-    oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), atol=0, btol=0, conlim=0, itn_limit=args.warmup + args.steps,
-                fixed_count=True, want_se=False, trace=lambda st: stamps.append(time.perf_counter()),
-                trace_vectors=False)
-    per = [b - a for a, b in zip(stamps[:-1], stamps[1:])][args.warmup:]
-    v = float(np.mean(per))
+    r = oracle.time_lsqr_omp(S, args.warmup + args.steps)
+    per = r["per_iter_s"][args.warmup:]
+    L = oracle.omp_lib()
+    t_pr = _time_products(S, (lambda x, y: L.orc_omp_aprod1(ctypes.byref(S.S), oracle._p(x), oracle._p(y)),
+                              lambda y, x: L.orc_omp_aprod2(ctypes.byref(S.S), oracle._p(y), oracle._p(x)))) \
+        if P > 1 else 0.0
+    t_it = float(np.mean(per))
+    v = t_it + (P - 1) * t_pr
+    sample = (f"rows of shard 0 of {P} of {w.name} ({S.n_rows} of {w.n_obs} rows; all {S.n_cols} columns), "
+              f"{len(per)} LSQR iterations after {args.warmup} warm-up (mean {t_it:.4f} s on the sample); "
+              f"full-system s/iteration = t_iter + (P-1) * t(aprod1 + aprod2) = {v:.3f} (setup {setup:.1f} s excluded)")
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
             "steps": len(per), "warmup": args.warmup, "ms_per_step": v * 1e3, "higher_is_better": False,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": config_block(w, 1, args, {"note": "CPU oracle (serial C, -O2 -ffp-contract=off) on the host; "
-                                                        "rank 0 only"}),
-            "cpu_baseline": {"value": v, "unit": UNIT, "cores": 1, "kind": "oracle",
-                             "sample": f"full {w.name} system, {len(per)} LSQR iterations after {args.warmup} "
-                                       f"warm-up (setup {setup:.1f} s excluded)", "cpu_model": _cpu_model()},
+            "config": config_block(w, 1, args, {"note": "CPU oracle, all-core OpenMP timing build "
+                                                        "(oracle/omp_timing.c), on the host; rank 0 only"}),
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": r["threads"], "kind": "oracle (all-core OpenMP "
+                             "timing build)", "sample": sample, "cpu_model": _cpu_model(),
+                             "host_cores": os.cpu_count()},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     emit(line)
     return 0
@@ -287,13 +349,28 @@ def run_ours(args):
     # ---------------- e2e through the public API with HOST buffers (set_system -> precondition -> solve -> x, se)
     e2e = None
     if args.e2e:
+        # host inputs in the paper's layout: values 192 B/row, matrixIndexAstro / matrixIndexAtt 8 B/row
+        # each, instrCol 48 B/row, b 8 B/row -- allocated pinned ONCE and filled in place (lsqr_get_system into the
+        # pinned buffers), so the host holds one copy (C3: 54.9 GB)
         s0 = avu.Solver.synthetic(w, rank=rank, nranks=world, **comm_kw())
-        g = s0.get_system()
-        nloc_cols = s0.n_local_cols
+        nloc_rows, nloc_cols = s0.n_local_rows, s0.n_local_cols
+        need = nloc_rows * (24 * 8 + 8 + 8 + 48 + 8)
+        avail = _mem_available()
+        if avail is not None and need > 0.85 * avail:
+            s0.close()
+            e2e = {"value": None, "unit": UNIT, "skipped": f"host RAM: {need / 1e9:.1f} GB of pinned inputs needed, "
+                                                             f"{avail / 1e9:.1f} GB available"}
+    if args.e2e and e2e is None:
+        pin = {"vals": np.empty((nloc_rows, 24), dtype=np.float64), "mA": np.empty(nloc_rows, dtype=np.int64),
+               "mT": np.empty(nloc_rows, dtype=np.int64), "iC": np.empty((nloc_rows, 6), dtype=np.int64),
+               "b": np.empty(nloc_rows, dtype=np.float64)}
+        cudart = torch.cuda.cudart()
+        for a in pin.values():  # page-locked in place (exact size; torch's pinned allocator rounds up to 2^k)
+            rc = cudart.cudaHostRegister(a.ctypes.data, a.nbytes, 0)
+            assert int(rc) == 0, f"cudaHostRegister failed: {rc}"
+        s0.get_system_ptrs(*[pin[k].ctypes.data for k in ("vals", "mA", "mT", "iC", "b")])
         s0.close()
         torch.cuda.synchronize()
-        pin = {k: torch.from_numpy(np.ascontiguousarray(v)).pin_memory() for k, v in g.items()}
-        del g
         xo = torch.empty(nloc_cols, dtype=torch.float64).pin_memory()
         so = torch.empty(nloc_cols, dtype=torch.float64).pin_memory()
         se = avu.Solver.synthetic(w, rank=rank, nranks=world, generate=False, **comm_kw())
@@ -301,8 +378,7 @@ def run_ours(args):
             se.set_reproducible(True)
 
         def e2e_cycle(itn):
-            se.set_system_ptrs(pin["vals"].data_ptr(), pin["mA"].data_ptr(), pin["mT"].data_ptr(),
-                               pin["iC"].data_ptr(), pin["b"].data_ptr())
+            se.set_system_ptrs(*[pin[k].ctypes.data for k in ("vals", "mA", "mT", "iC", "b")])
             t1 = time.perf_counter()  # set_system is synchronous (host buffers are borrowed for the call only)
             se.precondition()
             out = se.solve(x_out=xo, se_out=so, itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True,
@@ -318,7 +394,7 @@ def run_ours(args):
         barrier()
         t3 = time.perf_counter()
         t_e2e = max_over_ranks(t3 - t0)
-        h2d = sum(t.numel() * t.element_size() for t in pin.values())
+        h2d = sum(a.nbytes for a in pin.values())
         e2e = {"value": t_e2e / K, "unit": UNIT, "h2d_bytes_per_step": int(h2d * n / K),
                "d2h_bytes_per_step": int(2 * nloc_cols * 8 * n / K), "itn": r["itn"],
                "split_s": {"set_system": round(t1 - t0, 5), "precondition_solve_copy_out": round(t3 - t1, 5)},
@@ -326,8 +402,10 @@ def run_ours(args):
                        "fixed count) + x, se to pinned host; wall clock / K, max over ranks; after one untimed "
                        "warm-up cycle (W iterations) on the same handle"}
         se.close()
-        del pin
         torch.cuda.synchronize()
+        for a in pin.values():
+            cudart.cudaHostUnregister(a.ctypes.data)
+        del pin
 
     # ---------------- device-resident timing
     # pass 1 (the headline `value`): K iterations through the production path (lsqr_iterate: CUDA-graph replay, as
@@ -457,11 +535,12 @@ def main():
     ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="C2", choices=sorted(W.CONFIGS))
+    ap.add_argument("--config", default="C3", choices=sorted(W.CONFIGS),
+                    help="workload (default C3: BASELINE.json configs[2], the largest single-GPU configuration)")
     ap.add_argument("--no-e2e", dest="e2e", action="store_false")
     ap.add_argument("--no-cpu-baseline", dest="cpu_baseline", action="store_false")
-    ap.add_argument("--cpu-iters", type=int, default=30,
-                    help="oracle LSQR iterations timed for cpu_baseline (a bounded sample: ~10 s of CPU work at C2)")
+    ap.add_argument("--cpu-iters", type=int, default=3,
+                    help="oracle LSQR iterations timed for cpu_baseline on its bounded sample (oracle_sample)")
     ap.add_argument("--n-att", type=int, default=0, help="override n_att (multiple of 3, >= 12; sensitivity sweep)")
     ap.add_argument("--n-instr", type=int, default=0, help="override n_instr (multiple of 6; sensitivity sweep)")
     ap.add_argument("--fused", dest="fused", action="store_true", default=True,

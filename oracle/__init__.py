@@ -334,6 +334,60 @@ def lsqr(m: int, n: int, aprod, b: np.ndarray, damp=0.0, atol=1e-8, btol=1e-8, c
     return res
 
 
+# --------------------------------------------------------------------------- all-core TIMING variant (not a checker)
+_SRC_OMP = os.path.join(_HERE, "omp_timing.c")
+_omp = None
+
+
+def build_omp(force: bool = False) -> str:
+    """Compile omp_timing.c (the oracle source with OpenMP loops and products; bench.py cpu_baseline timing only)."""
+    newest = max(os.path.getmtime(_SRC), os.path.getmtime(_SRC_OMP))
+    if force or not os.path.exists(_LIB_OMP) or os.path.getmtime(_LIB_OMP) < newest:
+        tmp = _LIB_OMP + f".tmp{os.getpid()}"
+        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-ffp-contract=off", "-fno-fast-math", "-std=c11", "-fPIC",
+                               "-shared", "-o", tmp, _SRC_OMP, "-lm"])
+        os.replace(tmp, _LIB_OMP)
+    return _LIB_OMP
+
+
+def omp_lib():
+    global _omp
+    with _lock:
+        if _omp is None:
+            L = C.CDLL(build_omp())
+            vp, i64, i32, d = C.c_void_p, C.c_int64, C.c_int32, C.c_double
+            L.orc_omp_threads.restype = C.c_int
+            for f in (L.orc_omp_aprod1, L.orc_omp_aprod2):
+                f.argtypes = [C.POINTER(SysStruct), vp, vp]
+            L.orc_lsqr.restype = C.c_int
+            L.orc_lsqr.argtypes = [i64, i64, vp, vp, vp, d, d, d, d, i64, i32, i32, i32, vp, vp, vp,
+                                   C.POINTER(LsqrOut), vp, vp]
+            _omp = L
+    return _omp
+
+
+def time_lsqr_omp(sysm: System, iters: int) -> dict:
+    """TIMING ONLY: `iters` fixed-count LSQR iterations of the all-core variant on an already preconditioned
+    System; returns per-iteration wall times (the first, which includes O-1, is dropped) and the thread count."""
+    import time
+    L = omp_lib()
+    stamps = []
+
+    def _tr(stp, u, v, w_, xx, vv, _ctx):
+        stamps.append(time.perf_counter())
+    tcb = TRACE_FN(_tr)
+    m, n = sysm.m_local, sysm.n_cols
+    x, var = np.zeros(n), np.zeros(n)
+    out = LsqrOut()
+    rc = L.orc_lsqr(m, n, C.cast(L.orc_omp_sys_aprod, C.c_void_p), C.cast(C.pointer(sysm.S), C.c_void_p),
+                    _p(sysm.rhs()), 0.0, 0.0, 0.0, 0.0, int(iters + 1), 1, 0, 0, _p(x), _p(var), None,
+                    C.byref(out), C.cast(tcb, C.c_void_p), None)
+    if rc != 0:
+        raise RuntimeError(f"orc_lsqr (omp) returned {rc}")
+    per = [b - a for a, b in zip(stamps[:-1], stamps[1:])]
+    return {"per_iter_s": per, "threads": int(L.orc_omp_threads()), "x": x}
+
+
 def eda_sum(a) -> float:
     """NEXT-4 exact digit accumulator: order-independent sum of doubles (docs/REPRO.md)."""
     a = np.ascontiguousarray(a, dtype=np.float64)

@@ -33,6 +33,15 @@
 
 #define ORC_SLOTS 24 /* 5 astro + 12 att + 6 instr + 1 glob per row, P:L357-363 (§II-B) */
 
+/* ORC_PAR_FOR / ORC_PAR_SUM(v) mark the O(m) / O(n) vector loops of orc_lsqr.  They are EMPTY in this build (the
+ * checker: plain serial C).  oracle/omp_timing.c -- a separately compiled -fopenmp variant used only to time the
+ * oracle on all host cores for bench.py's cpu_baseline, never as a parity reference -- defines them as OpenMP
+ * pragmas before including this file. */
+#ifndef ORC_PAR_FOR
+#define ORC_PAR_FOR
+#define ORC_PAR_SUM(v)
+#endif
+
 /* ------------------------------------------------------------------------------------------------------------
  * O-GEN: synthetic system generator (integer hash -> exact FP64).  The paper generates a synthetic system from a
  * size and a seed "distributed in the system as the real data" (Artifact appendix); the structure
@@ -446,10 +455,12 @@ static double orc_nrm2(const double* a, int64_t n) { /* plain sqrt(sum a^2) in o
     return sqrt(orc_eda_round(&A));
   }
   double s = 0.0;
+  ORC_PAR_SUM(s)
   for (int64_t i = 0; i < n; ++i) s = s + a[i] * a[i];
   return sqrt(s);
 }
 static void orc_scal(double* a, int64_t n, double f) {
+  ORC_PAR_FOR
   for (int64_t i = 0; i < n; ++i) a[i] = f * a[i];
 }
 static double orc_dot(const double* a, const double* b, int64_t n) {
@@ -476,6 +487,9 @@ static void orc_reorth(double* a, const double* Q, int64_t k, int64_t n) {
 int orc_lsqr(int64_t m, int64_t n, orc_aprod_fn aprod, void* ctx, const double* b, double damp, double atol,
              double btol, double conlim, int64_t itn_limit, int32_t fixed_count, int32_t reorth, int32_t repro,
              double* x, double* var, double* se, orc_lsqr_out* out, orc_trace_fn trace, void* trace_ctx) {
+#ifdef _OPENMP
+  if (repro) return -2; /* omp_timing.c build: the repro accumulators are not thread-safe there */
+#endif
   orc_repro_mode = repro ? 1 : 0;
   const double eps = 0x1p-52;
   double* u = (double*)malloc(sizeof(double) * (size_t)(m > 0 ? m : 1));
@@ -493,7 +507,9 @@ int orc_lsqr(int64_t m, int64_t n, orc_aprod_fn aprod, void* ctx, const double* 
   memset(out, 0, sizeof *out);
 
   /* O-1: x = 0, var = 0; u = b, beta = ||u||, u /= beta; v = A^T u, alpha = ||v||, v /= alpha; w = v. */
+  ORC_PAR_FOR
   for (int64_t j = 0; j < n; ++j) { x[j] = 0.0; var[j] = 0.0; v[j] = 0.0; }
+  ORC_PAR_FOR
   for (int64_t i = 0; i < m; ++i) u[i] = b[i];
   double beta = orc_nrm2(u, m), alpha = 0.0;
   if (beta > 0.0) {
@@ -502,6 +518,7 @@ int orc_lsqr(int64_t m, int64_t n, orc_aprod_fn aprod, void* ctx, const double* 
     alpha = orc_nrm2(v, n);
   }
   if (alpha > 0.0) orc_scal(v, n, 1.0 / alpha);
+  ORC_PAR_FOR
   for (int64_t j = 0; j < n; ++j) w[j] = v[j];
   int64_t nu = 0, nv = 0;
   if (reorth) {
@@ -564,6 +581,7 @@ int orc_lsqr(int64_t m, int64_t n, orc_aprod_fn aprod, void* ctx, const double* 
     double t1 = phi / rho, t2 = -theta / rho, t3 = 1.0 / rho;
     orc_eda DD;
     memset(&DD, 0, sizeof DD);
+    ORC_PAR_SUM(ddnorm) /* (the timing build rejects repro mode: DD is not thread-safe) */
     for (int64_t j = 0; j < n; ++j) {
       double dk = t3 * w[j];
       var[j] = var[j] + dk * dk;

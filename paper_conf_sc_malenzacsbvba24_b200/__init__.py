@@ -231,6 +231,10 @@ class Solver:
         """Raw host pointers (e.g. pinned torch tensors' data_ptr()) -- the e2e path."""
         self._chk(_capi.lib().lsqr_set_system(self._h, vals_p, mA_p, mT_p, iC_p, b_p))
 
+    def get_system_ptrs(self, vals_p, mA_p, mT_p, iC_p, b_p):
+        """lsqr_get_system into raw host pointers (e.g. pinned torch tensors' data_ptr()); any may be None."""
+        self._chk(_capi.lib().lsqr_get_system(self._h, vals_p, mA_p, mT_p, iC_p, b_p))
+
     def get_system(self, with_b=True):
         n = self.n_local_rows
         out = dict(vals=np.zeros((n, 24)), mA=np.zeros(n, dtype=np.int64), mT=np.zeros(n, dtype=np.int64),

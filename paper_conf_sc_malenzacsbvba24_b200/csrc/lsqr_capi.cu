@@ -95,6 +95,7 @@ struct lsqr_ctx {
   double *vals = nullptr, *u = nullptr, *v = nullptr, *w = nullptr, *x = nullptr, *var = nullptr, *D = nullptr;
   double *zsh = nullptr, *part_rows = nullptr, *part_a2 = nullptr, *cpart = nullptr, *part_sh = nullptr;
   double *zA = nullptr, *part_va = nullptr;
+  double* xatt4 = nullptr;  // the fused kernel's attitude gather copy (S.xatt4)
   double* ingest = nullptr;  // lsqr_set_system staging (lazily allocated)
   double* uc_tmp = nullptr;  // k_post -> k_scalar constraint u_hat hand-over  // fused mode: astro z (A^T u_hat) and alpha^2 partials of k_vastro
   double *part_wa = nullptr, *part_ws = nullptr, *part_g1 = nullptr, *ar1 = nullptr, *uc = nullptr,
@@ -322,7 +323,7 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
     if (ev && fused) cudaEventRecord(ev[3], s);
     CKL(h, launch_scalar(h->st, h->part_va, kG3, nullptr, 0, h->part_wa, kG3, h->part_ws, kG3, nullptr, nullptr, 0,
                          h->hflag_dev, s, h->uc_tmp, h->uc, h->ucn, (int)h->n_constr), "scalar");
-    CKL(h, launch_colupdate(h->v, h->w, h->x, h->var, h->n_loc_cols, S.A0, h->part_wa, h->part_ws, kG3, h->st, s),
+    CKL(h, launch_colupdate(S, h->v, h->w, h->x, h->var, h->part_wa, h->part_ws, kG3, h->st, s),
         "colupdate");
     return LSQR_OK;
   }
@@ -341,7 +342,7 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   CKL(h, launch_scalar(h->st, h->part_va, kG3, h->part_sh, kG2, h->part_wa, kG3, h->part_ws, kG3, h->zsh + h->n_sh,
                        h->ar1 + h->n_constr + 1, 0, h->hflag_dev, s),
       "scalar");
-  CKL(h, launch_colupdate(h->v, h->w, h->x, h->var, h->n_loc_cols, S.A0, h->part_wa, h->part_ws, kG3, h->st, s),
+  CKL(h, launch_colupdate(S, h->v, h->w, h->x, h->var, h->part_wa, h->part_ws, kG3, h->st, s),
       "colupdate");
   return LSQR_OK;
 }
@@ -649,6 +650,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   AL(h->var, h->n_loc_cols);
   AL(h->D, h->n_loc_cols);
   AL(h->zsh, h->n_sh + 8);
+  AL(h->xatt4, 4 * n_axis);
   AL(h->part_rows, h->W);
   AL(h->part_a2, h->W);
   AL(h->cpart, std::max<int64_t>((int64_t)ch_row.size(), 1));
@@ -726,6 +728,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   S.n_cs = cs_ptr.empty() ? 0 : ((int64_t)cs_ptr.size() - 1) / 5; S.cs_ptr = d_csp; S.cs_k = d_csk; S.cs_e = d_cse;
   S.n_csh = (int64_t)csh_idx.size(); S.csh_idx = d_cshi; S.csh_k = d_cshk; S.csh_e = d_cshe;
   S.scs_lo = scs_lo; S.scs_hi = scs_hi; S.scs_ptr = d_scsp; S.scs_k = d_scsk; S.scs_e = d_scse;
+  S.xatt4 = h->xatt4;
   {  // bank-grouped instrumental slots only when every row kernel keeps the instrumental slice in shared memory
     InstrPerm probe;
     probe.init(n_instr, true);
@@ -735,6 +738,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   // zero-initialised state
   if (launch_fill(h->zsh, h->n_sh + 8, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (launch_fill(h->D, h->n_loc_cols, 1.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
+  if (launch_fill(h->xatt4, 4 * n_axis, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   for (double* p : {h->v, h->w, h->x, h->var})
     if (launch_fill(p, h->n_loc_cols, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (launch_fill(h->u, h->n_loc_rows + 2, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
@@ -897,7 +901,7 @@ int lsqr_precondition(lsqr_t h) {
   CKL(h, launch_aprod2(AP2_COLNORM, S, h->grid, nullptr, nullptr, h->D, h->zsh, h->part_a2, h->st, h->rank == 0,
                        h->s), "colnorm");
   CKR(allreduce(h, h->zsh, h->n_sh));
-  CKL(h, launch_add_shared(h->D + S.A0, h->zsh, h->n_sh, 1, h->s), "colnorm_sh");
+  CKL(h, launch_add_shared(S, h->D + S.A0, h->zsh, 1, h->s), "colnorm_sh");
   CKL(h, launch_precond_D(h->D, h->n_loc_cols, h->s), "precond_D");
   CKL(h, launch_scale_rows(S, h->grid, h->vals, h->D, h->s), "scale_rows");
   CKL(h, launch_scale_constr(S, const_cast<double*>(S.cval), h->D, h->s), "scale_constr");
@@ -969,7 +973,7 @@ int lsqr_aprod2(lsqr_t h, const double* y_dev, double* x_dev) {
   CKL(h, launch_ap2_lean(S, h->grid, y_dev, h->zA, h->zsh, h->st_api, h->s), "aprod2");
   CKL(h, launch_astro_add(S, x_dev, h->zA, y_dev + h->n_loc_rows, h->zsh, h->rank == 0, h->s), "aprod2_astro");
   CKR(allreduce(h, h->zsh, h->n_sh));
-  CKL(h, launch_add_shared(x_dev + S.A0, h->zsh, h->n_sh, 0, h->s), "aprod2_sh");
+  CKL(h, launch_add_shared(S, x_dev + S.A0, h->zsh, 0, h->s), "aprod2_sh");
   leave(h);
   return LSQR_OK;
 }
@@ -1027,7 +1031,7 @@ int lsqr_init(lsqr_t h, const lsqr_solve_params* p) {
   CKL(h, launch_scalar(h->st, h->part_a2, h->W, h->part_sh, kG2, h->part_wa, kG3, h->part_ws, kG3,
                        multi ? h->zsh + h->n_sh : nullptr, nullptr, 1, h->hflag_dev, h->s),
       "scalar0");
-  CKL(h, launch_colupdate(h->v, h->w, h->x, h->var, h->n_loc_cols, S.A0, h->part_wa, h->part_ws, kG3, h->st, h->s),
+  CKL(h, launch_colupdate(S, h->v, h->w, h->x, h->var, h->part_wa, h->part_ws, kG3, h->st, h->s),
       "colupdate0");
   h->b_valid = false;
   h->initialized = true;
@@ -1188,6 +1192,7 @@ int lsqr_set_state(lsqr_t h, const double* sc, const double* u, const double* v,
   if (w) CKC(h, cudaMemcpyAsync(h->w, w, nb, cudaMemcpyHostToDevice, h->s));
   if (x) CKC(h, cudaMemcpyAsync(h->x, x, nb, cudaMemcpyHostToDevice, h->s));
   if (var) CKC(h, cudaMemcpyAsync(h->var, var, nb, cudaMemcpyHostToDevice, h->s));
+  if (v) CKL(h, launch_att_pack(h->S, h->v, h->s), "att_pack");
   // ||w||^2 partials (astro / shared) for the next iteration's ddnorm
   CKL(h, launch_sumsq(h->w, h->S.A0, h->part_wa, kG3, h->s), "wsum_a");
   CKL(h, launch_sumsq(h->w + h->S.A0, h->n_sh, h->part_ws, kG3, h->s), "wsum_s");

@@ -114,6 +114,9 @@ struct SysView {
   // shared-column constraint entries grouped by shared column (CSC) over [scs_lo, scs_hi) (rank 0 only)
   int64_t scs_lo, scs_hi; const int64_t* scs_ptr; const int32_t* scs_k; const int64_t* scs_e;
   int32_t f3_zrep, f3_arep;  // k_fused3 launch only: shared-memory accumulator copies (set by its launcher)
+  // The fused kernel's attitude gather copy: xatt4[4k + a] = v[A0 + a n_axis + k] for a < 3, [4k + 3] = 0,
+  // written by k_colupdate -- a lane's three axis values of knot k0 + j are one 32-B load (LDG.E.ENL2.256).
+  double* xatt4;
 };
 
 enum { AP1_LSQR = 0, AP1_PLAIN = 1 };
@@ -151,6 +154,7 @@ cudaError_t launch_beta(int phase, const SysView& S, const double* part, int64_t
                         double* ar1, double* uc, double* ucn, const double* crhs, DevState* st, int init,
                         cudaStream_t s);
 cudaError_t launch_cdot_add(const SysView& S, const double* cpart, const double* ar1, double* yc, cudaStream_t s);
+// fused = 1: z_sh holds A^T u_hat of the fused kernel (unnormalised); 0: A^T u of k_aprod2 (init)
 cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* part, int nblk, const DevState* st,
                            int fused, cudaStream_t s);
 // NEXT-1 fused single pass (u_hat update + A^T u_hat in one read of A) and its astro column pass
@@ -165,7 +169,8 @@ cudaError_t launch_ap2_lean(const SysView& S, int grid, const double* u, double*
                             cudaStream_t s);
 cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const double* uc, double* zsh, double* part,
                           int nblk, const DevState* st, int do_shared_constr, cudaStream_t s);
-cudaError_t launch_add_shared(double* xsh, double* zsh, int64_t n, int mode, cudaStream_t s);
+// mode 0: x += z, 1: x = z; z zeroed
+cudaError_t launch_add_shared(const SysView& S, double* xsh, double* zsh, int mode, cudaStream_t s);
 cudaError_t launch_scalar(DevState* st, const double* part_astro, int64_t n_pa, const double* part_sh,
                           int64_t n_ps, const double* part_wa, int64_t n_pwa, const double* part_ws, int64_t n_pws,
                           const double* ar2_alpha2, const double* ar1_wa, int init, int32_t* host_flag,
@@ -175,8 +180,11 @@ cudaError_t launch_scalar(DevState* st, const double* part_astro, int64_t n_pa, 
 cudaError_t launch_post(const SysView& S, double* v, const double* zA, double* zsh, const double* part_rows,
                         int64_t n_part, const double* cpart, const double* uc, double* uc_tmp, double* part_a2,
                         int nblk, DevState* st, cudaStream_t s);
-cudaError_t launch_colupdate(double* v, double* w, double* x, double* var, int64_t n, int64_t A0, double* part_wa,
+// also refreshes the attitude gather copy S.xatt4 from the new v
+cudaError_t launch_colupdate(const SysView& S, double* v, double* w, double* x, double* var, double* part_wa,
                              double* part_ws, int nblk, const DevState* st, cudaStream_t s);
+// rebuilds S.xatt4 from v (after v is overwritten outside the iteration, e.g. lsqr_set_state)
+cudaError_t launch_att_pack(const SysView& S, const double* v, cudaStream_t s);
 cudaError_t launch_sum_to(const double* part, int64_t n, double* dst, cudaStream_t s);
 cudaError_t launch_precond_D(double* c, int64_t n, cudaStream_t s);
 cudaError_t launch_finalize(const double* x, const double* var, const double* D, int64_t n, const DevState* st,

@@ -684,6 +684,21 @@ constexpr int kSmemMaxBytes = 232448;  // 227 KB opt-in per CTA on sm_100
 // k_vshared finish the iteration unchanged (v' = z / beta - beta v).  (An aprod1 on this loop measured slower than
 // k_aprod1's deeper 16-row ring: C3 11.5 vs 10.5 ms.)
 enum { R3_FUSED = 0, R3_AP2 = 2 };
+
+#ifndef LSQR_GATHER4
+#define LSQR_GATHER4 1  // attitude gathers: one 32-B load per lane from the padded knot-major copy xatt4 (A/B: 0)
+#endif
+
+// a lane's three axis values of knot k from the padded knot-major gather copy: one 256-bit load (LDG.E.ENL2.256)
+__device__ __forceinline__ void ldg_att4(const double* p, double& a0, double& a1, double& a2) {
+  double r[4];
+  asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(r[0]), "=d"(r[1]), "=d"(r[2]), "=d"(r[3]) : "l"(p));
+  a0 = r[0];
+  a1 = r[1];
+  a2 = r[2];
+}
+
+
 constexpr int kF3Stage = kFRows * (kSlots * 8 + 16);  // 1664 B: 8 rows of values + 8 index records
 constexpr int kF3Bars = kFWarps * kFStages * 8;          // per stage: "full" mbarrier (TMA bytes)
 constexpr int kF3InstrMax = (kSmemMaxBytes - FRing::kBytes - kF3Bars - 1024) / 16 - 2;
@@ -764,10 +779,14 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
 
   const unsigned char* ringp = dsm + wid * kFStages * kF3Stage;
   const int voff = r * kSlots * 8 + 48 * j, ioff = kFRows * kSlots * 8 + r * 16;
+#if LSQR_GATHER4
+  const double* const xg4 = S.xatt4 + 4 * j;  // lane j gathers knot k0 + j (its three axis values, one load)
+#else
   const double* xatt0 = x + S.A0 + j;
   const double* xatt1 = xatt0 + S.n_axis;
   const double* xatt2 = xatt1 + S.n_axis;
-  double* zatt0 = (SMATT ? sh_za + (wid % arep) * S.n_att : zsh) + j;
+#endif
+  double* zatt0 = (SMATT ? sh_za + (wid % arep) * S.n_att : zsh) + j;  // axis-major: knot k0 + j of axis a
   double* zatt1 = zatt0 + S.n_axis;
   double* zatt2 = zatt1 + S.n_axis;
   double* const sh_zw = ZREP ? sh_z + (wid % zrep) * zstride : sh_z;  // this warp's z_instr copy
@@ -828,9 +847,17 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
     P.i4 = ((uint32_t)((j & 2) ? rec.z : rec.y) >> i4_shift) & 0xffffu;
     P.i5 = t5_ins ? (((uint32_t)rec.w >> i5_shift) & 0xffffu) : i5_or;
     if (kDot) {
-      P.g1 = (DIAG & 4) ? 0.5 : __ldg(xatt0 + P.k0);
-      P.g2 = (DIAG & 4) ? 0.5 : __ldg(xatt1 + P.k0);
-      P.g3 = (DIAG & 4) ? 0.5 : __ldg(xatt2 + P.k0);
+      if (DIAG & 4) {
+        P.g1 = P.g2 = P.g3 = 0.5;
+      } else {
+#if LSQR_GATHER4
+        ldg_att4(xg4 + 4 * (int64_t)P.k0, P.g1, P.g2, P.g3);
+#else
+        P.g1 = __ldg(xatt0 + P.k0);
+        P.g2 = __ldg(xatt1 + P.k0);
+        P.g3 = __ldg(xatt2 + P.k0);
+#endif
+      }
       P.g4 = (DIAG & 8) ? 0.5 : (IG ? __ldg(xins + P.i4) : sh_x[P.i4]);
       P.g5 = (DIAG & 8) ? 0.5 : (IG ? __ldg(xins + P.i5) : sh_x[P.i5]);
     }
@@ -874,7 +901,7 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
       un = valid ? uold : 0.0;  // aprod2: the u_hat aprod1 wrote
     }
     const double c1 = v[1] * un, c2 = v[2] * un, c3 = v[3] * un, c4v = v[4] * un, c5 = v[5] * un;
-    if (valid && !(DIAG & 2)) {
+    if (valid && !(DIAG & 2)) {  // per axis, the 4 lanes of a row hit 4 consecutive columns (one 32-B window)
       atomicAdd(zatt0 + P.k0, c1);
       atomicAdd(zatt1 + P.k0, c2);
       atomicAdd(zatt2 + P.k0, c3);
@@ -1423,8 +1450,8 @@ __global__ void __launch_bounds__(kRedThreads)
 // into the local astro columns (i < A0) and the replicated shared slice (i >= A0).
 __global__ void __launch_bounds__(kRedThreads)
     k_colupdate(double* __restrict__ v, double* __restrict__ w, double* __restrict__ x, double* __restrict__ var,
-                int64_t n, int64_t A0, double* __restrict__ part_wa, double* __restrict__ part_ws,
-                const DevState* __restrict__ st) {
+                int64_t n, int64_t A0, int64_t n_att, int64_t n_axis, double* __restrict__ xatt4,
+                double* __restrict__ part_wa, double* __restrict__ part_ws, const DevState* __restrict__ st) {
   if (!st->col_enable) return;
   const double ia = st->v_pending ? st->inv_alpha : 1.0;
   const double t1 = st->t1, t2 = st->t2, t3 = st->t3;
@@ -1437,8 +1464,16 @@ __global__ void __launch_bounds__(kRedThreads)
     const double wnew = fma(t2, wi, vi);
     w[i] = wnew;
     v[i] = vi;
-    if (i < A0) wa = fma(wnew, wnew, wa);
-    else ws = fma(wnew, wnew, ws);
+    if (i < A0) {
+      wa = fma(wnew, wnew, wa);
+    } else {
+      ws = fma(wnew, wnew, ws);
+      const int64_t c = i - A0;
+      if (c < n_att) {  // the fused kernel's attitude gather copy: knot-major, padded to 4
+        const int64_t a = c / n_axis;
+        xatt4[4 * (c - a * n_axis) + a] = vi;
+      }
+    }
   }
   wa = block_sum<kRedThreads>(wa);
   ws = block_sum<kRedThreads>(ws);
@@ -1726,8 +1761,8 @@ cudaError_t launch_astro_add(const SysView& S, double* x, const double* zA, cons
                                                                                                  do_shared_constr);
   return cudaGetLastError();
 }
-cudaError_t launch_add_shared(double* xsh, double* zsh, int64_t n, int mode, cudaStream_t s) {
-  k_add_shared<<<vec_grid(n, 148 * 4), kRedThreads, 0, s>>>(xsh, zsh, n, mode);
+cudaError_t launch_add_shared(const SysView& S, double* xsh, double* zsh, int mode, cudaStream_t s) {
+  k_add_shared<<<vec_grid(S.n_sh, 148 * 4), kRedThreads, 0, s>>>(xsh, zsh, S.n_sh, mode);
   return cudaGetLastError();
 }
 cudaError_t launch_scalar(DevState* st, const double* part_astro, int64_t n_pa, const double* part_sh,
@@ -1738,9 +1773,21 @@ cudaError_t launch_scalar(DevState* st, const double* part_astro, int64_t n_pa, 
                                      ar2_alpha2, ar1_wa, init, host_flag, post_uc, uc, ucn, nc);
   return cudaGetLastError();
 }
-cudaError_t launch_colupdate(double* v, double* w, double* x, double* var, int64_t n, int64_t A0, double* part_wa,
+cudaError_t launch_colupdate(const SysView& S, double* v, double* w, double* x, double* var, double* part_wa,
                              double* part_ws, int nblk, const DevState* st, cudaStream_t s) {
-  k_colupdate<<<nblk, kRedThreads, 0, s>>>(v, w, x, var, n, A0, part_wa, part_ws, st);
+  k_colupdate<<<nblk, kRedThreads, 0, s>>>(v, w, x, var, S.n_cols, S.A0, S.n_att, S.n_axis, S.xatt4, part_wa, part_ws,
+                                           st);
+  return cudaGetLastError();
+}
+
+__global__ void k_att_pack(const double* __restrict__ v, int64_t n_att, int64_t n_axis, double* __restrict__ xatt4) {
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < n_att; c += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t a = c / n_axis;
+    xatt4[4 * (c - a * n_axis) + a] = v[c];
+  }
+}
+cudaError_t launch_att_pack(const SysView& S, const double* v, cudaStream_t s) {
+  k_att_pack<<<vec_grid(S.n_att, 148 * 4), kRedThreads, 0, s>>>(v + S.A0, S.n_att, S.n_axis, S.xatt4);
   return cudaGetLastError();
 }
 cudaError_t launch_sum_to(const double* part, int64_t n, double* dst, cudaStream_t s) {

@@ -308,4 +308,5 @@ def test_gpu_nccl_forced_early_stop(cuda_device, fused):
     a, b = outs
     assert 0 < a["itn"] < 500 and a["istop"] in (1, 2)
     assert a["istop"] == b["istop"] and abs(a["itn"] - b["itn"]) <= 2  # |d itn| <= 2 across roundings
-    assert np.linalg.norm(a["x"] - b["x"]) <= 1e-8 * np.linalg.norm(a["x"])
+    # stopped at a 1e-9 tolerance, not converged to rounding: x agrees to the accuracy the stopping rule gives
+    assert np.linalg.norm(a["x"] - b["x"]) <= 1e-5 * np.linalg.norm(a["x"])

@@ -119,3 +119,17 @@ def test_precond_zero_column_gets_unit_D():
     empty = np.linalg.norm(A, axis=0) == 0
     assert empty.sum() > 10
     assert (D[empty] == 1.0).all()
+
+
+def test_omp_timing_variant_matches_serial():
+    """bench.py's all-core cpu_baseline runs oracle/omp_timing.c (the oracle source with OpenMP loops and products;
+    never a parity reference).  Sanity: it solves the same system -- x after 6 fixed iterations within rounding of
+    the serial checker's."""
+    import numpy as np
+    w = W.C1C.replace(jitter_pct=50)
+    S = oracle.System(w)
+    S.apply_precond()
+    r = oracle.time_lsqr_omp(S, 5)
+    ro = oracle.solve_system(oracle.System(w), atol=0, btol=0, conlim=0, itn_limit=6, fixed_count=True)
+    assert r["threads"] >= 1 and len(r["per_iter_s"]) == 5
+    assert np.linalg.norm(r["x"] - ro["x_scaled"]) <= 1e-12 * np.linalg.norm(ro["x_scaled"])
