@@ -177,8 +177,8 @@ def cpu_baseline(w, iters=3, repro=False, all_cores=True):
         omp = {"value": o_it + (P - 1) * o_pr, "cores": r["threads"], "sample_s_per_iter": o_it,
                "sample_products_s": o_pr,
                "build": "oracle/omp_timing.c (the oracle source with OpenMP loops/products; timing only)"}
-        out.update(value=omp["value"], cores=omp["cores"], kind="oracle (all-core OpenMP timing build)",
-                   all_cores=omp)
+        out.update(value=omp["value"], cores=omp["cores"], build="all-core OpenMP timing build (value, cores); "
+                   "the serial checker as it stands under 'serial'", all_cores=omp)
     return out
 
 
@@ -294,9 +294,9 @@ def run_reference(args):
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": config_block(w, 1, args, {"note": "CPU oracle, all-core OpenMP timing build "
                                                         "(oracle/omp_timing.c), on the host; rank 0 only"}),
-            "cpu_baseline": {"value": v, "unit": UNIT, "cores": r["threads"], "kind": "oracle (all-core OpenMP "
-                             "timing build)", "sample": sample, "cpu_model": _cpu_model(),
-                             "host_cores": os.cpu_count()},
+            "cpu_baseline": {"value": v, "unit": UNIT, "cores": r["threads"], "kind": "oracle",
+                             "build": "all-core OpenMP timing build (oracle/omp_timing.c)", "sample": sample,
+                             "cpu_model": _cpu_model(), "host_cores": os.cpu_count()},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     emit(line)
     return 0
