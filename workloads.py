@@ -69,7 +69,11 @@ C4 = Workload("C4", n_stars=4_000_000, n_obs=780_000_000, n_att=3_000_000, n_ins
 C5 = Workload("C5", n_stars=3_125_000, n_obs=625_000_000, n_att=3_000_000, n_instr=6_000, jitter_pct=50,
               n_ext_stars=1_000, seed=TIMING_SEED)
 
-CONFIGS = {w.name: w for w in (C1, C1C, C2, C3, C4, C5)}
+# C4's shape (n_att = 3,000,000: the 24 MB shared slice AR2 carries) at 1/100 of its stars and rows: the strong-scaling
+# flow of bench.py at test size (--scaling strong --config C4s)
+C4S = C4.replace(name="C4s", n_stars=40_000, n_obs=7_800_000)
+
+CONFIGS = {w.name: w for w in (C1, C1C, C2, C3, C4, C4S, C5)}
 
 
 def micro(n_stars=7, obs=30, n_att=24, n_instr=12, n_glob=1, jitter=50, n_ext=0, seed=3, **kw) -> Workload:
