@@ -163,7 +163,8 @@ def cpu_baseline(w, iters=3, repro=False, all_cores=True):
     t_pr = _time_products(S, (S.aprod1_repro, S.aprod2_repro) if repro else (S.aprod1, S.aprod2)) if P > 1 else 0.0
     serial = {"value": t_it + (P - 1) * t_pr, "cores": 1, "sample_s_per_iter": t_it, "sample_products_s": t_pr}
     sample = (f"rows of shard 0 of {P} of {w.name} ({S.n_rows} of {w.n_obs} rows; all {S.n_cols} columns), "
-              f"{len(per)} timed LSQR iterations after 1 untimed; full-system s/iteration extrapolated as "
+              f"{len(per)} timed LSQR iterations{' (repro mode)' if repro else ''} after 1 untimed; "
+              f"full-system s/iteration extrapolated as "
               f"t_iter + (P-1) * t(aprod1 + aprod2) on the sample (setup {t_setup:.1f} s excluded)")
     out = {"value": serial["value"], "unit": UNIT, "cores": 1, "kind": "oracle",
            "sample": sample, "serial": serial, "cpu_model": _cpu_model(), "host_cores": os.cpu_count()}
