@@ -359,11 +359,18 @@ def run_ours(args):
         s0 = avu.Solver.synthetic(w, rank=rank, nranks=world, **comm_kw())
         nloc_rows, nloc_cols = s0.n_local_rows, s0.n_local_cols
         need = nloc_rows * (24 * 8 + 8 + 8 + 48 + 8)
+        local_ranks = int(os.environ.get("LOCAL_WORLD_SIZE", "1"))  # ranks of this node pin their inputs at once
         avail = _mem_available()
-        if avail is not None and need > 0.85 * avail:
+        short = avail is not None and need * local_ranks > 0.85 * avail
+        if multi:  # the decision must be the same on every rank (the e2e leg has barriers and reductions)
+            t = torch.tensor([1.0 if short else 0.0], dtype=torch.float64, device="cuda" if use_nccl else "cpu")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            short = bool(t.item() > 0)
+        if short:
             s0.close()
-            e2e = {"value": None, "unit": UNIT, "skipped": f"host RAM: {need / 1e9:.1f} GB of pinned inputs needed, "
-                                                             f"{avail / 1e9:.1f} GB available"}
+            e2e = {"value": None, "unit": UNIT,
+                   "skipped": f"host RAM: {need * local_ranks / 1e9:.1f} GB of pinned inputs needed on this node, "
+                              f"{(avail or 0) / 1e9:.1f} GB available"}
     if args.e2e and e2e is None:
         pin = {"vals": np.empty((nloc_rows, 24), dtype=np.float64), "mA": np.empty(nloc_rows, dtype=np.int64),
                "mT": np.empty(nloc_rows, dtype=np.int64), "iC": np.empty((nloc_rows, 6), dtype=np.int64),

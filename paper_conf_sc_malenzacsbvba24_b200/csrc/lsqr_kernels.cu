@@ -685,6 +685,12 @@ constexpr int kSmemMaxBytes = 232448;  // 227 KB opt-in per CTA on sm_100
 // k_aprod1's deeper 16-row ring: C3 11.5 vs 10.5 ms.)
 enum { R3_FUSED = 0, R3_AP2 = 2 };
 
+#ifndef LSQR_IDX32
+#define LSQR_IDX32 0    // index record as one 4-B shared load per lane + quad shuffles (A/B: 1.5-2.5 % slower at C2)
+#endif
+#ifndef LSQR_T5PRED
+#define LSQR_T5PRED 1   // slot t=5 gathers only on the instrumental lanes (1, 2); v_glob from a register (lane 3)
+#endif
 #ifndef LSQR_GATHER4
 #define LSQR_GATHER4 1  // attitude gathers: one 32-B load per lane from the padded knot-major copy xatt4 (A/B: 0)
 #endif
@@ -795,6 +801,7 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
   // lane 3 gathers v_glob (slot nsl; IG: column G0 = I0 + n_instr, which exists iff n_glob); lane 0 ignores its g5
   const uint32_t i5_or = (j == 3) ? (IG ? (S.n_glob ? (uint32_t)S.n_instr : 0u) : (uint32_t)nsl) : 0u;
   const double* const xins = x + S.I0;
+  const double vglob_r = (kDot && S.n_glob) ? __ldg(x + S.G0) : 0.0;
   const int i4_shift = (j & 1) << 4;
   double* const urow = u + r_lo + r;
 
@@ -842,10 +849,22 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
   auto prefetch = [&](int q, int sl, Pre& P) {
     mbar_wait(bar + 8 * sl, (uint32_t)(q >> 2) & 1u);
     static_assert(kFStages == 4, "parity uses q / 4");
+#if LSQR_IDX32
+    // lane j of a row reads word j of the row's 16-B record (k0, ic01, ic23, ic45): one conflict-free 128-B
+    // wavefront per group; the quad exchanges the words it needs
+    const uint32_t wj = *reinterpret_cast<const uint32_t*>(ringp + sl * kF3Stage + ioff + 4 * j);
+    const int qb = lane & ~3;
+    P.k0 = __shfl_sync(0xffffffffu, (int)wj, qb);
+    const uint32_t w4 = __shfl_sync(0xffffffffu, wj, qb + 1 + (j >> 1));
+    const uint32_t w5 = __shfl_sync(0xffffffffu, wj, qb + 3);
+    P.i4 = (w4 >> i4_shift) & 0xffffu;
+    P.i5 = t5_ins ? ((w5 >> i5_shift) & 0xffffu) : i5_or;
+#else
     const int4 rec = *reinterpret_cast<const int4*>(ringp + sl * kF3Stage + ioff);
     P.k0 = rec.x;
     P.i4 = ((uint32_t)((j & 2) ? rec.z : rec.y) >> i4_shift) & 0xffffu;
     P.i5 = t5_ins ? (((uint32_t)rec.w >> i5_shift) & 0xffffu) : i5_or;
+#endif
     if (kDot) {
       if (DIAG & 4) {
         P.g1 = P.g2 = P.g3 = 0.5;
@@ -859,7 +878,13 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
 #endif
       }
       P.g4 = (DIAG & 8) ? 0.5 : (IG ? __ldg(xins + P.i4) : sh_x[P.i4]);
+#if LSQR_T5PRED
+      if (DIAG & 8) P.g5 = 0.5;
+      else if (t5_ins) P.g5 = IG ? __ldg(xins + P.i5) : sh_x[P.i5];
+      else P.g5 = vglob_r;  // lane 3: v_glob; lane 0 uses the astro value instead
+#else
       P.g5 = (DIAG & 8) ? 0.5 : (IG ? __ldg(xins + P.i5) : sh_x[P.i5]);
+#endif
     }
   };
 

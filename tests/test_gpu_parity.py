@@ -163,6 +163,20 @@ def rel(a, b):
     return np.linalg.norm(a - b) / max(np.linalg.norm(b), 1e-300)
 
 
+def identical_inputs(S, w, vals_gpu, D_gpu):
+    """The oracle system scaled exactly as the GPU scaled its own (the GPU's scaled values; constraint values times
+    the GPU's D, as k_scale_constr does), so both iterate on bit-identical inputs and differ only in the iteration's
+    rounding (a perturbation of the matrix itself, ~1 ulp from a differently rounded D, also moves the trajectory)."""
+    S.apply_precond()
+    S.vals[:] = vals_gpu
+    c_raw = oracle.constraints(w)
+    if c_raw is not None:
+        S.c_val[:] = c_raw[2] * D_gpu[S.c_col]
+    S.D = D_gpu.copy()
+    S._mk_struct()
+    return S
+
+
 def permuted_control(S, perm):
     """Control run of SURVEY §8(c): the same system with its rows in the order `perm` (new row i = old row perm[i])
     and the constraint entries of each row reversed -- every sum of the products in a different order.  Returns the
@@ -195,9 +209,7 @@ def free_run_curves(avu, w, kmax=30, fused=False, n_controls=5):
     kmax]), plus the oracle run (100 iterations)."""
     s = gpu_solver(avu, w)
     s.precondition()
-    S = oracle.System(w)
-    S.apply_precond()
-    S.vals[:] = s.get_system(with_b=False)["vals"]   # both sides on the GPU's scaled matrix (identical inputs)
+    S = identical_inputs(oracle.System(w), w, s.get_system(with_b=False)["vals"], s.get_precond())
     res_o, hist = oracle_trace(S, 100, atol=0, btol=0, conlim=0)
     n = S.n_rows
     ctrl = []
@@ -264,11 +276,11 @@ SIGMA_CASES = [(W.C1, 60, 1e-2, True), (W.C1, 100, 1e-2, False), (W.C1C, 80, 1e-
 def test_sigma_statistical(avu, w, itn, ceil, strict, fused):
     s = gpu_solver(avu, w)
     s.precondition()
-    out = s.solve(itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True, fused=fused)
     D = s.get_precond()
+    Ag = s.get_system(with_b=False)["vals"]
+    out = s.solve(itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True, fused=fused)
     s.close()
-    S = oracle.System(w)
-    S.apply_precond()
+    S = identical_inputs(oracle.System(w), w, Ag, D)
     ro = oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), atol=0, btol=0, conlim=0, itn_limit=itn, fixed_count=True)
     dc = []
     for p in control_perms(S.n_rows, 8):
@@ -290,9 +302,7 @@ def test_lsqr_teacher_forced_step(avu, w, fused):
     k = 1..59, vectors u, v, w, x, var and the scalars of the recurrence."""
     s = gpu_solver(avu, w)
     s.precondition()
-    S = oracle.System(w)
-    S.apply_precond()
-    S.vals[:] = s.get_system(with_b=False)["vals"]
+    S = identical_inputs(oracle.System(w), w, s.get_system(with_b=False)["vals"], s.get_precond())
     _, hist = oracle_trace(S, 60, atol=0, btol=0, conlim=0)
     s.init(itn_limit=1000, atol=0, btol=0, conlim=0, fixed_count=True, fused=fused)
     for k in range(1, 60):
@@ -325,9 +335,7 @@ def test_lsqr_teacher_forced_step_C2(avu, fused):
     ks = (1, 2, 3, 5, 8, 13, 21, 34)
     s = gpu_solver(avu, w)
     s.precondition()
-    S = oracle.System(w)
-    S.apply_precond()
-    S.vals[:] = s.get_system(with_b=False)["vals"]
+    S = identical_inputs(oracle.System(w), w, s.get_system(with_b=False)["vals"], s.get_precond())
     keep = set(ks) | {k + 1 for k in ks}
     hist = {}
 
@@ -346,9 +354,7 @@ def test_lsqr_solve_api_and_stopping(avu):
     w = W.C1
     s = gpu_solver(avu, w)
     s.precondition()
-    S = oracle.System(w)
-    S.apply_precond()
-    S.vals[:] = s.get_system(with_b=False)["vals"]
+    S = identical_inputs(oracle.System(w), w, s.get_system(with_b=False)["vals"], s.get_precond())
     ro = oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), atol=1e-10, btol=1e-10, itn_limit=500)
     out = s.solve(itn_limit=500, atol=1e-10, btol=1e-10)
     assert out["istop"] == ro["istop"] and abs(out["itn"] - ro["itn"]) <= 2
