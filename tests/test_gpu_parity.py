@@ -258,22 +258,22 @@ def test_lsqr_free_run_and_converged(avu, w, fused):
     s.close()
 
 
-# sigma (O-4) is an estimate whose value depends on the rounding trajectory (SURVEY EXP-4/5).  Measured
-# (tests/tools/sigma_study.py, profiles/round2/sigma_study.txt): on C1 the median relative sigma difference between
-# two valid roundings grows exponentially with the iteration count once the Ritz values converge -- ~3e-15 at k = 20,
-# 1e-14 at 40, 5e-11 at 60, 1e-6 at 80, 1e-5..1e-3 at 100 -- for reordered-sum oracle controls and GPU runs alike
-# (the GPU's own run-to-run spread at k = 100 is 6e-5..1e-3: atomics order).  With the constraint rows (C1c) sigma
-# moves in steps: a lost-orthogonality "ghost" direction re-enters var at an iteration that depends on the rounding,
-# shifting EVERY sigma by the same ~0.4-1 % (k = 100: 7 of 8 oracle reorderings 4.4e-3, the 8th 4.0e-4; k = 90:
-# 3e-7..2e-3; k = 80: 7e-6..7e-5).  So the paper's statistical criterion is applied strictly --
-# median difference <= 2x the median of 8 controls and <= 1e-2 -- at iterations where the valid roundings agree
-# (C1 at k = 60, C1c at k = 80), and at the paper's k = 100 as a bound on the step (<= 1e-2 on C1, <= 2e-2 on C1c).
-SIGMA_CASES = [(W.C1, 60, 1e-2, True), (W.C1, 100, 1e-2, False), (W.C1C, 80, 1e-2, True), (W.C1C, 100, 2e-2, False)]
+# sigma (O-4) is an estimate whose value depends on the rounding trajectory (SURVEY EXP-4/5; DESIGN R5).  Measured
+# (tests/tools/sigma_study.py, tests/tools/ortho_study.py, profiles/round2/): once the Ritz values converge, the
+# Lanczos vectors lose orthogonality, and "ghost" directions re-enter var -- how early depends on the size of the
+# rounding errors.  The GPU's tree/FMA reductions lose orthogonality ~100x more slowly than the oracle's sequential
+# sums (C1, k = 81: max |v_k . v_j| 2.5e-6 fused / 3.4e-5 two-pass vs 8.7e-4 oracle), so past k ~ 70 the GPU's sigma
+# departs from the oracle's (C1, k = 100: ~1e-3) while reordered-sum oracle controls, which lose orthogonality like
+# the oracle, stay closer to it (~1e-5).  The reference that does not depend on the rounding is the oracle's test-only
+# fully reorthogonalised LSQR (pinned to the OLS formula at k = n, tests/test_oracle_lsqr.py): the GPU's sigma must
+# be no farther from it than the controls are (it is usually closer), and where no ghost has appeared yet (C1, k = 60)
+# it must also agree with the oracle's like a control does (<= 2x the controls' median, <= 1e-2: SURVEY 8(c)).
+SIGMA_CASES = [(W.C1, 60, True), (W.C1, 100, False), (W.C1C, 60, False), (W.C1C, 100, False)]
 
 
 @pytest.mark.parametrize("fused", [False, True], ids=["twopass", "fused"])
-@pytest.mark.parametrize("w,itn,ceil,strict", SIGMA_CASES, ids=["C1-k60", "C1-k100", "C1c-k80", "C1c-k100"])
-def test_sigma_statistical(avu, w, itn, ceil, strict, fused):
+@pytest.mark.parametrize("w,itn,vs_oracle", SIGMA_CASES, ids=["C1-k60", "C1-k100", "C1c-k60", "C1c-k100"])
+def test_sigma_statistical(avu, w, itn, vs_oracle, fused):
     s = gpu_solver(avu, w)
     s.precondition()
     D = s.get_precond()
@@ -281,18 +281,20 @@ def test_sigma_statistical(avu, w, itn, ceil, strict, fused):
     out = s.solve(itn_limit=itn, atol=0, btol=0, conlim=0, fixed_count=True, fused=fused)
     s.close()
     S = identical_inputs(oracle.System(w), w, Ag, D)
-    ro = oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), atol=0, btol=0, conlim=0, itn_limit=itn, fixed_count=True)
-    dc = []
-    for p in control_perms(S.n_rows, 8):
-        C = permuted_control(S, p)
-        rc = oracle.lsqr(C.m_local, C.n_cols, C, C.rhs(), atol=0, btol=0, conlim=0, itn_limit=itn,
-                         fixed_count=True)
-        dc.append(np.median(np.abs(rc["se"] / ro["se"] - 1)))
-    d = np.median(np.abs((out["se"] / D) / ro["se"] - 1))
-    print(f"\nse at k={itn}: median rel diff gpu {d:.2e}; controls " + " ".join(f"{c:.1e}" for c in dc))
-    assert d <= ceil
-    if strict:
-        assert d <= 2 * np.median(dc), (d, dc)
+    kw = dict(atol=0, btol=0, conlim=0, itn_limit=itn, fixed_count=True)
+    ro = oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), **kw)
+    rr = oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), reorth=True, **kw)
+    ses = [oracle.lsqr(C.m_local, C.n_cols, C, C.rhs(), **kw)["se"]
+           for C in (permuted_control(S, p) for p in control_perms(S.n_rows, 6))]
+    med = lambda a, b: float(np.median(np.abs(a / b - 1)))
+    se_g = out["se"] / D
+    d_or, dc_or = med(se_g, ro["se"]), [med(c, ro["se"]) for c in ses]
+    d_re, dc_re = med(se_g, rr["se"]), [med(c, rr["se"]) for c in ses] + [med(ro["se"], rr["se"])]
+    print(f"\nse at k={itn}: vs oracle gpu {d_or:.2e} controls " + " ".join(f"{c:.1e}" for c in dc_or)
+          + f" | vs reorthogonalised gpu {d_re:.2e} oracle+controls " + " ".join(f"{c:.1e}" for c in dc_re))
+    assert d_re <= max(2 * np.median(dc_re), 1e-12), (d_re, dc_re)
+    if vs_oracle:
+        assert d_or <= 1e-2 and d_or <= 2 * np.median(dc_or), (d_or, dc_or)
 
 
 @pytest.mark.parametrize("fused", [False, True], ids=["twopass", "fused"])
