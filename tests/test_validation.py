@@ -31,6 +31,11 @@ def reference():
     S = oracle.System(W_VAL)
     r = oracle.solve_system(S, itn_limit=3000, fixed_count=False, **TOL)
     assert r["istop"] in (1, 2, 4, 5), r["istop"]
+    # the rounding-independent sigma at the same iteration: the oracle's test-only fully reorthogonalised LSQR
+    # (pinned to the OLS formula at k = n, tests/test_oracle_lsqr.py); DESIGN R5
+    rr = oracle.lsqr(S.m_local, S.n_cols, S, S.rhs(), reorth=True, atol=0, btol=0, conlim=0, itn_limit=r["itn"],
+                     fixed_count=True)
+    r["se_reorth"] = S.D * rr["se"]
     return r
 
 
@@ -40,7 +45,7 @@ def paper_criteria(x, se, x_ref, se_ref):
     return within.mean(), float(np.mean(dsig)), float(np.std(dsig))
 
 
-def check(tag, out, x_ref, se_ref, itn_ref, x_tol=1e-8):
+def check(tag, out, x_ref, se_ref, itn_ref, x_tol=1e-8, se_reorth=None):
     frac, mean_d, std_d = paper_criteria(out["x"], out["se"], x_ref, se_ref)
     print(f"\nvalidation {tag}: itn {out['itn']} (oracle {itn_ref}), istop {out['istop']}; "
           f"x within 1 sigma: {100 * frac:.3f} %; sigma diff mean {mean_d:.2e} std {std_d:.2e}; "
@@ -48,9 +53,16 @@ def check(tag, out, x_ref, se_ref, itn_ref, x_tol=1e-8):
     assert out["istop"] in (1, 2, 4, 5)
     assert abs(out["itn"] - itn_ref) <= max(5, itn_ref // 20)
     assert frac == 1.0
-    # the LSQR sigma is itself an estimate whose value depends on the iteration's rounding history (SURVEY EXP-4,
-    # EXP-5); the paper's criterion is statistical
-    assert abs(mean_d) <= 2e-2 and std_d <= 5e-2
+    # The LSQR sigma is itself an estimate that depends on the iteration's rounding history (SURVEY EXP-4/5, DESIGN
+    # R5): at this early convergence (k ~ 30-40) the oracle's sigma is 13 % below the reorthogonalised value (C2val),
+    # and two valid roundings differ by ~2 % on average.  The paper's criterion is statistical: mean and spread of
+    # the sigma differences small against sigma itself.
+    assert abs(mean_d) <= 5e-2 and std_d <= 5e-2
+    if se_reorth is not None:  # and the GPU's sigma is no farther from the rounding-independent value than the oracle's
+        dg = np.median(np.abs(out["se"] / se_reorth - 1))
+        do = np.median(np.abs(se_ref / se_reorth - 1))
+        print(f"  sigma vs reorthogonalised: gpu {dg:.3e}, oracle {do:.3e}")
+        assert dg <= 1.25 * do
     assert np.linalg.norm(out["x"] - x_ref) <= x_tol * np.linalg.norm(x_ref)
 
 
@@ -61,7 +73,8 @@ def test_validation_vs_oracle(cuda_device, reference, fused):
     s.precondition()
     out = s.solve(itn_limit=3000, fused=fused, **TOL)
     s.close()
-    check(f"C2val fused={fused}", out, reference["x"], reference["se"], reference["itn"])
+    check(f"C2val fused={fused}", out, reference["x"], reference["se"], reference["itn"],
+          se_reorth=reference["se_reorth"])
 
 
 @pytest.mark.parametrize("name", ["C3v", "C3"])
@@ -147,7 +160,8 @@ def test_validation_across_ranks(cuda_device, reference, P):
     assert len(itns) == 1, itns  # every rank stopped at the same iteration
     itn, istop = itns.pop()
     out = dict(x=x, se=se, itn=itn, istop=istop)
-    check(f"C2val P={P} vs oracle", out, reference["x"], reference["se"], reference["itn"])
+    check(f"C2val P={P} vs oracle", out, reference["x"], reference["se"], reference["itn"],
+          se_reorth=reference["se_reorth"])
     s = avu.Solver.synthetic(w)
     s.precondition()
     one = s.solve(itn_limit=3000, **TOL)
