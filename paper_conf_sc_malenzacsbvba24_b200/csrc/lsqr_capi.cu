@@ -95,7 +95,8 @@ struct lsqr_ctx {
   double *vals = nullptr, *u = nullptr, *v = nullptr, *w = nullptr, *x = nullptr, *var = nullptr, *D = nullptr;
   double *zsh = nullptr, *part_rows = nullptr, *part_a2 = nullptr, *cpart = nullptr, *part_sh = nullptr;
   double *zA = nullptr, *part_va = nullptr;
-  double* xatt4 = nullptr;  // the fused kernel's attitude gather copy (S.xatt4)
+  double* xatt4 = nullptr;      // the attitude gather copy of v (S.xatt4), kept by k_colupdate
+  double* xatt4_api = nullptr;  // lsqr_aprod1's gather copy of its x (allocated on first use; pad entries unused)
   double* ingest = nullptr;  // lsqr_set_system staging (lazily allocated)
   double* uc_tmp = nullptr;  // k_post -> k_scalar constraint u_hat hand-over  // fused mode: astro z (A^T u_hat) and alpha^2 partials of k_vastro
   double *part_wa = nullptr, *part_ws = nullptr, *part_g1 = nullptr, *ar1 = nullptr, *uc = nullptr,
@@ -307,7 +308,7 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   if (fused) {
     CKL(h, launch_fused(S, h->grid, h->v, h->u, h->zA, h->zsh, h->part_rows, h->cpart, h->st, s), "fused");
   } else {
-    CKL(h, launch_aprod1(AP1_LSQR, S, h->grid, h->v, h->u, h->part_rows, h->cpart, h->st, s), "aprod1");
+    CKL(h, launch_aprod1(AP1_LSQR, S, h->grid, h->v, h->u, h->part_rows, h->cpart, h->st, s, h->xatt4), "aprod1");
   }
   if (ev) cudaEventRecord(ev[1], s);
   if (!fused) {
@@ -666,7 +667,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   AL(h->ucn, nc + 1);
   AL(h->crhs, nc + 1);
   AL(h->tmp, std::max<int64_t>(h->n_loc_cols, nc + 1));
-  AL(h->tmax, 8);
+  AL(h->tmax, std::max<int32_t>(h->nranks, 8));
   AL(h->st, 1);
   AL(h->st_api, 1);
   double* d_cval = nullptr;
@@ -948,7 +949,11 @@ int lsqr_aprod1(lsqr_t h, const double* x_dev, double* y_dev) {
   if (!h->have_system) return fail(h, LSQR_ESTATE, "no system");
   SysView& S = h->S;
   enter(h);
-  CKL(h, launch_aprod1(AP1_PLAIN, S, h->grid, x_dev, y_dev, h->part_rows, h->cpart, h->st, h->s), "aprod1");
+  // the attitude slice of x in the padded knot-major layout (32 B per knot, <= 32 MB), then one 256-bit load per lane
+  if (!h->xatt4_api) CKR(dalloc(h, &h->xatt4_api, 4 * h->n_axis));
+  CKL(h, launch_att_pack(S, x_dev, h->s, h->xatt4_api), "att_pack");
+  CKL(h, launch_aprod1(AP1_PLAIN, S, h->grid, x_dev, y_dev, h->part_rows, h->cpart, h->st, h->s, h->xatt4_api),
+      "aprod1");
   if (h->n_constr > 0) {
     if (!h->multi) {
       CKL(h, launch_cdot_add(S, h->cpart, nullptr, y_dev + h->n_loc_rows, h->s), "cdot");
@@ -1248,15 +1253,16 @@ int lsqr_solve(lsqr_t h, const lsqr_solve_params* p, lsqr_result* res, double* x
   if (res) {
     res->t_iter_mean_s = res->itn > 0 ? ms * 1e-3 / res->itn : 0.0;
     res->t_iter_max_over_ranks_s = res->t_iter_mean_s;
-    if (h->multi && h->comm_kind == LSQR_COMM_NCCL) {
-      double t = res->t_iter_mean_s;
-      CKC(h, cudaMemcpyAsync(h->tmax, &t, sizeof t, cudaMemcpyHostToDevice, h->s));
-      ncclResult_t r = g_nccl.AllReduce(h->tmax, h->tmax, 1, ncclFloat64, ncclMax, h->nccl, h->s);
-      if (r != ncclSuccess) return fail(h, LSQR_ENCCL, "ncclAllReduce(max)");
+    if (h->multi) {
+      // max over ranks through the communicator's SUM allreduce (NCCL or the host callback): every rank puts its
+      // time in its own slot of an nranks-long vector of zeros
+      std::vector<double> tv(h->nranks, 0.0);
+      tv[h->rank] = res->t_iter_mean_s;
+      CKC(h, cudaMemcpyAsync(h->tmax, tv.data(), sizeof(double) * h->nranks, cudaMemcpyHostToDevice, h->s));
+      CKR(allreduce(h, h->tmax, h->nranks));
+      CKC(h, cudaMemcpyAsync(tv.data(), h->tmax, sizeof(double) * h->nranks, cudaMemcpyDeviceToHost, h->s));
       CKC(h, cudaStreamSynchronize(h->s));
-      CKC(h, cudaMemcpyAsync(&t, h->tmax, sizeof t, cudaMemcpyDeviceToHost, h->s));
-      CKC(h, cudaStreamSynchronize(h->s));
-      res->t_iter_max_over_ranks_s = t;
+      res->t_iter_max_over_ranks_s = *std::max_element(tv.begin(), tv.end());
     }
   }
   return LSQR_OK;

@@ -141,8 +141,9 @@ cudaError_t launch_ingest(const double* sv, const int64_t* smA, const int64_t* s
                           int64_t nrows, const int64_t* star_ptr, int64_t n_stars_loc, int64_t star_begin,
                           int64_t A0g, int64_t I0g, int64_t n_axis, int64_t n_instr, InstrPerm ip, double* vals,
                           IdxRec* idx, unsigned long long* err, cudaStream_t s);
+// xg4: the padded knot-major copy of x's attitude slice (launch_att_pack), or nullptr (gathers from x)
 cudaError_t launch_aprod1(int mode, const SysView& S, int grid, const double* x, double* y, double* part,
-                          double* cpart, const DevState* st, cudaStream_t s);
+                          double* cpart, const DevState* st, cudaStream_t s, const double* xg4 = nullptr);
 cudaError_t launch_aprod2(int mode, const SysView& S, int grid, const double* y, const double* ucn, double* xv,
                           double* zsh, double* part, const DevState* st, int do_shared_constr, cudaStream_t s);
 cudaError_t launch_scale_rows(const SysView& S, int grid, double* vals, const double* D, cudaStream_t s);
@@ -183,8 +184,8 @@ cudaError_t launch_post(const SysView& S, double* v, const double* zA, double* z
 // also refreshes the attitude gather copy S.xatt4 from the new v
 cudaError_t launch_colupdate(const SysView& S, double* v, double* w, double* x, double* var, double* part_wa,
                              double* part_ws, int nblk, const DevState* st, cudaStream_t s);
-// rebuilds S.xatt4 from v (after v is overwritten outside the iteration, e.g. lsqr_set_state)
-cudaError_t launch_att_pack(const SysView& S, const double* v, cudaStream_t s);
+// the padded knot-major copy of v's attitude slice into dst (nullptr: S.xatt4, e.g. after lsqr_set_state)
+cudaError_t launch_att_pack(const SysView& S, const double* v, cudaStream_t s, double* dst = nullptr);
 cudaError_t launch_sum_to(const double* part, int64_t n, double* dst, cudaStream_t s);
 cudaError_t launch_precond_D(double* c, int64_t n, cudaStream_t s);
 cudaError_t launch_finalize(const double* x, const double* var, const double* D, int64_t n, const DevState* st,

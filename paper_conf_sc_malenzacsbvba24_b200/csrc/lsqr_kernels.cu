@@ -354,14 +354,25 @@ __device__ __forceinline__ void smem_add_n(double* const (&a)[N], const double (
   }
 }
 
+// a lane's three axis values of knot k from the padded knot-major gather copy: one 256-bit load (LDG.E.ENL2.256)
+__device__ __forceinline__ void ldg_att4(const double* p, double& a0, double& a1, double& a2) {
+  double r[4];
+  asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(r[0]), "=d"(r[1]), "=d"(r[2]), "=d"(r[3]) : "l"(p));
+  a0 = r[0];
+  a1 = r[1];
+  a2 = r[2];
+}
+
 // ------------------------------------------------------------------------------------------------ aprod1
 // MODE AP1_LSQR:  u_hat[i] = sum_s a_is v[col_is] - u_scale * u_hat[i];  per-warp partial of u_hat^2 (beta^2).
 // MODE AP1_PLAIN: y[i] += sum_s a_is x[col_is].
 // Constraint rows: per-chunk partial dots of the owned entries -> cpart (combined by k_beta / k_cdot).
-template <int MODE, bool SMEM_INSTR>
+// G4: the attitude values come from a padded knot-major copy of x (xg4[4k + a]): one 256-bit load per
+// lane instead of three gathers.
+template <int MODE, bool SMEM_INSTR, bool G4 = false>
 __global__ void __launch_bounds__(kThreads, 1)
     k_aprod1(SysView S, const double* __restrict__ x, double* __restrict__ y, double* __restrict__ part,
-             double* __restrict__ cpart, const DevState* __restrict__ st) {
+             double* __restrict__ cpart, const DevState* __restrict__ st, const double* __restrict__ xg4) {
   extern __shared__ __align__(128) unsigned char dsm[];
   if (MODE == AP1_LSQR && st->halted) return;
   // the instrumental slice of x (<= 64 KB) is staged in shared memory: its gathers are random and L1-hostile
@@ -413,9 +424,13 @@ __global__ void __launch_bounds__(kThreads, 1)
       // only the attitude values are gathered from global memory (L2) per row; instr from shared memory
       const int k0 = valid[q] ? rec.k0 : 0;
       xv[q][0] = ac.cj;
-      xv[q][1] = __ldg(xatt0 + k0);
-      xv[q][2] = __ldg(xatt1 + k0);
-      xv[q][3] = __ldg(xatt2 + k0);
+      if (G4) {
+        ldg_att4(xg4 + 4 * ((int64_t)k0 + j), xv[q][1], xv[q][2], xv[q][3]);
+      } else {
+        xv[q][1] = __ldg(xatt0 + k0);
+        xv[q][2] = __ldg(xatt1 + k0);
+        xv[q][3] = __ldg(xatt2 + k0);
+      }
       const uint32_t i4 = valid[q] ? ic4_of(rec, j) : 0u, i5 = valid[q] ? ic5_of(rec, j) : 0u;
       xv[q][4] = SMEM_INSTR ? xins[i4] : __ldg(xins + i4);
       const double a_ins = SMEM_INSTR ? xins[i5] : __ldg(xins + i5);
@@ -695,14 +710,6 @@ enum { R3_FUSED = 0, R3_AP2 = 2 };
 #define LSQR_GATHER4 1  // attitude gathers: one 32-B load per lane from the padded knot-major copy xatt4 (A/B: 0)
 #endif
 
-// a lane's three axis values of knot k from the padded knot-major gather copy: one 256-bit load (LDG.E.ENL2.256)
-__device__ __forceinline__ void ldg_att4(const double* p, double& a0, double& a1, double& a2) {
-  double r[4];
-  asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(r[0]), "=d"(r[1]), "=d"(r[2]), "=d"(r[3]) : "l"(p));
-  a0 = r[0];
-  a1 = r[1];
-  a2 = r[2];
-}
 
 
 constexpr int kF3Stage = kFRows * (kSlots * 8 + 16);  // 1664 B: 8 rows of values + 8 index records
@@ -1624,23 +1631,29 @@ static cudaError_t ensure_smem(const void* fn, size_t bytes) {
   return e;
 }
 
-template <int MODE, bool SM>
+template <int MODE, bool SM, bool G4>
 static cudaError_t ap1(const SysView& S, int grid, const double* x, double* y, double* part, double* cpart,
-                       const DevState* st, cudaStream_t s) {
+                       const DevState* st, const double* xg4, cudaStream_t s) {
   const size_t smem = kRingBytes + kBarBytes + (SM ? (size_t)S.ip.slots() * sizeof(double) : 0);
-  cudaError_t e = ensure_smem((const void*)k_aprod1<MODE, SM>, smem);
+  cudaError_t e = ensure_smem((const void*)k_aprod1<MODE, SM, G4>, smem);
   if (e != cudaSuccess) return e;
-  k_aprod1<MODE, SM><<<grid, kThreads, smem, s>>>(S, x, y, part, cpart, st);
+  k_aprod1<MODE, SM, G4><<<grid, kThreads, smem, s>>>(S, x, y, part, cpart, st, xg4);
   return cudaGetLastError();
 }
 
 cudaError_t launch_aprod1(int mode, const SysView& S, int grid, const double* x, double* y, double* part,
-                          double* cpart, const DevState* st, cudaStream_t s) {
+                          double* cpart, const DevState* st, cudaStream_t s, const double* xg4) {
   const bool sm = S.ip.slots() <= kInstrSmemMax;
-  if (mode == AP1_LSQR) return sm ? ap1<AP1_LSQR, true>(S, grid, x, y, part, cpart, st, s)
-                                  : ap1<AP1_LSQR, false>(S, grid, x, y, part, cpart, st, s);
-  return sm ? ap1<AP1_PLAIN, true>(S, grid, x, y, part, cpart, st, s)
-            : ap1<AP1_PLAIN, false>(S, grid, x, y, part, cpart, st, s);
+  if (xg4) {  // the two products that run per iteration / per API call in the default regimes
+    if (mode == AP1_LSQR) return sm ? ap1<AP1_LSQR, true, true>(S, grid, x, y, part, cpart, st, xg4, s)
+                                    : ap1<AP1_LSQR, false, true>(S, grid, x, y, part, cpart, st, xg4, s);
+    return sm ? ap1<AP1_PLAIN, true, true>(S, grid, x, y, part, cpart, st, xg4, s)
+              : ap1<AP1_PLAIN, false, true>(S, grid, x, y, part, cpart, st, xg4, s);
+  }
+  if (mode == AP1_LSQR) return sm ? ap1<AP1_LSQR, true, false>(S, grid, x, y, part, cpart, st, nullptr, s)
+                                  : ap1<AP1_LSQR, false, false>(S, grid, x, y, part, cpart, st, nullptr, s);
+  return sm ? ap1<AP1_PLAIN, true, false>(S, grid, x, y, part, cpart, st, nullptr, s)
+            : ap1<AP1_PLAIN, false, false>(S, grid, x, y, part, cpart, st, nullptr, s);
 }
 
 template <int MODE, bool SM>
@@ -1818,8 +1831,8 @@ __global__ void k_att_pack(const double* __restrict__ v, int64_t n_att, int64_t 
     xatt4[4 * (c - a * n_axis) + a] = v[c];
   }
 }
-cudaError_t launch_att_pack(const SysView& S, const double* v, cudaStream_t s) {
-  k_att_pack<<<vec_grid(S.n_att, 148 * 4), kRedThreads, 0, s>>>(v + S.A0, S.n_att, S.n_axis, S.xatt4);
+cudaError_t launch_att_pack(const SysView& S, const double* v, cudaStream_t s, double* dst) {
+  k_att_pack<<<vec_grid(S.n_att, 148 * 4), kRedThreads, 0, s>>>(v + S.A0, S.n_att, S.n_axis, dst ? dst : S.xatt4);
   return cudaGetLastError();
 }
 cudaError_t launch_sum_to(const double* part, int64_t n, double* dst, cudaStream_t s) {

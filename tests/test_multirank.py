@@ -122,6 +122,10 @@ def _gpu_worker(rank, world, port, q, itn, fused):
         its = [None] * world
         dist_obj.all_gather_object(its, (early["itn"], early["istop"]))
         assert len(set(its)) == 1, its
+        # lsqr_result.t_iter_max_over_ranks_s: the max of every rank's mean iteration time (through the callback)
+        tms = [None] * world
+        dist_obj.all_gather_object(tms, (early["t_iter_mean_s"], early["t_iter_max_over_ranks_s"]))
+        assert all(t[1] == max(m for m, _ in tms) for t in tms), tms
         # plain products through the ABI
         xg = torch.ones(s.n_local_cols, dtype=torch.float64, device="cuda")
         yg = torch.zeros(s.n_local_rows + s.n_constr, dtype=torch.float64, device="cuda")
