@@ -8,6 +8,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -97,6 +98,7 @@ struct lsqr_ctx {
   double *zA = nullptr, *part_va = nullptr;
   double* xatt4 = nullptr;      // the attitude gather copy of v (S.xatt4), kept by k_colupdate
   double* xatt4_api = nullptr;  // lsqr_aprod1's gather copy of its x (allocated on first use; pad entries unused)
+  double* z4 = nullptr;         // attitude window accumulator of the fused kernel (S.z4), or nullptr
   double* ingest = nullptr;  // lsqr_set_system staging (lazily allocated)
   double* uc_tmp = nullptr;  // k_post -> k_scalar constraint u_hat hand-over  // fused mode: astro z (A^T u_hat) and alpha^2 partials of k_vastro
   double *part_wa = nullptr, *part_ws = nullptr, *part_g1 = nullptr, *ar1 = nullptr, *uc = nullptr,
@@ -350,8 +352,9 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
 
 int kernels_per_iteration(lsqr_t h) {
   if (h->repro) return h->multi ? 15 : 7;
-  if (!h->params.two_pass) return h->multi ? 9 : 4;
-  return h->multi ? 10 : 5;
+  const int fold = h->z4 ? 1 : 0;  // k_att_fold after the row pass
+  if (!h->params.two_pass) return (h->multi ? 9 : 4) + fold;
+  return (h->multi ? 10 : 5) + fold;
 }
 
 int build_graph(lsqr_t h) {
@@ -652,6 +655,8 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   AL(h->D, h->n_loc_cols);
   AL(h->zsh, h->n_sh + 8);
   AL(h->xatt4, 4 * n_axis);
+  const bool use_z4 = n_att > 4096 && n_att <= kZ4MaxAtt && !getenv("LSQR_NO_Z4");  // 4096: kSmAttMax (smem copies)
+  if (use_z4) AL(h->z4, 4 * n_att);
   AL(h->part_rows, h->W);
   AL(h->part_a2, h->W);
   AL(h->cpart, std::max<int64_t>((int64_t)ch_row.size(), 1));
@@ -730,6 +735,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   S.n_csh = (int64_t)csh_idx.size(); S.csh_idx = d_cshi; S.csh_k = d_cshk; S.csh_e = d_cshe;
   S.scs_lo = scs_lo; S.scs_hi = scs_hi; S.scs_ptr = d_scsp; S.scs_k = d_scsk; S.scs_e = d_scse;
   S.xatt4 = h->xatt4;
+  S.z4 = h->z4;
   {  // bank-grouped instrumental slots only when every row kernel keeps the instrumental slice in shared memory
     InstrPerm probe;
     probe.init(n_instr, true);
@@ -740,6 +746,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   if (launch_fill(h->zsh, h->n_sh + 8, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (launch_fill(h->D, h->n_loc_cols, 1.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (launch_fill(h->xatt4, 4 * n_axis, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
+  if (h->z4 && launch_fill(h->z4, 4 * n_att, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   for (double* p : {h->v, h->w, h->x, h->var})
     if (launch_fill(p, h->n_loc_cols, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (launch_fill(h->u, h->n_loc_rows + 2, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);

@@ -117,7 +117,16 @@ struct SysView {
   // The fused kernel's attitude gather copy: xatt4[4k + a] = v[A0 + a n_axis + k] for a < 3, [4k + 3] = 0,
   // written by k_colupdate -- a lane's three axis values of knot k0 + j are one 32-B load (LDG.E.ENL2.256).
   double* xatt4;
+  // Attitude window accumulator of the fused kernel, or nullptr: z4[a][k0][j] (4 doubles per window
+  // start k0, 32-B aligned) collects the 4 lanes' REDs of a row in one aligned sector; k_att_fold adds it into z_sh
+  // after each pass.  Used when 4 n_att doubles stay well inside L2 (n_att <= kZ4MaxAtt) and the attitude slice is
+  // not privatised in shared memory.
+  double* z4;
 };
+#ifndef LSQR_Z4_MAX_ATT
+#define LSQR_Z4_MAX_ATT (1 << 20)
+#endif
+constexpr int64_t kZ4MaxAtt = LSQR_Z4_MAX_ATT;
 
 enum { AP1_LSQR = 0, AP1_PLAIN = 1 };
 enum { AP2_LSQR = 0, AP2_PLAIN = 1, AP2_COLNORM = 2 };

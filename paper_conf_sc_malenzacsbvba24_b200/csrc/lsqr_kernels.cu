@@ -799,9 +799,13 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
   const double* xatt1 = xatt0 + S.n_axis;
   const double* xatt2 = xatt1 + S.n_axis;
 #endif
-  double* zatt0 = (SMATT ? sh_za + (wid % arep) * S.n_att : zsh) + j;  // axis-major: knot k0 + j of axis a
-  double* zatt1 = zatt0 + S.n_axis;
-  double* zatt2 = zatt1 + S.n_axis;
+  // attitude accumulator: axis-major z_att (lane j -> knot k0 + j of axis a), or, when S.z4 is set, the window
+  // accumulator z4[a][k0][j] (one 32-B-aligned sector per row and axis; folded into z_sh by k_att_fold)
+  const bool z4 = !SMATT && S.z4 != nullptr;
+  const int kmul = z4 ? 4 : 1;
+  double* zatt0 = (SMATT ? sh_za + (wid % arep) * S.n_att : (z4 ? S.z4 : zsh)) + j;
+  double* zatt1 = zatt0 + kmul * S.n_axis;
+  double* zatt2 = zatt1 + kmul * S.n_axis;
   double* const sh_zw = ZREP ? sh_z + (wid % zrep) * zstride : sh_z;  // this warp's z_instr copy
   const bool t5_ins = (j == 1 || j == 2);  // t=5 slot: lane 0 astro 4, lanes 1, 2 instr 4, 5, lane 3 global
   const int i5_shift = (j & 2) << 3;
@@ -934,9 +938,10 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
     }
     const double c1 = v[1] * un, c2 = v[2] * un, c3 = v[3] * un, c4v = v[4] * un, c5 = v[5] * un;
     if (valid && !(DIAG & 2)) {  // per axis, the 4 lanes of a row hit 4 consecutive columns (one 32-B window)
-      atomicAdd(zatt0 + P.k0, c1);
-      atomicAdd(zatt1 + P.k0, c2);
-      atomicAdd(zatt2 + P.k0, c3);
+      const int ko = kmul * P.k0;
+      atomicAdd(zatt0 + ko, c1);
+      atomicAdd(zatt1 + ko, c2);
+      atomicAdd(zatt2 + ko, c3);
     }
     if (valid && !(DIAG & 1)) {
       double* const zi = IG ? zsh + S.n_att : sh_zw;
@@ -1772,26 +1777,54 @@ static int diag_mode() {
 }
 #endif
 
+// z4 -> z_sh: z_att[a][k] += sum_j z4[a][k - j][j] (windows k - j in [0, n_axis - 4]); every z4 entry belongs to
+// exactly one column, which zeroes it after reading (the accumulator is clean for the next pass)
+__global__ void k_att_fold(double* __restrict__ z4, double* __restrict__ zsh, int64_t n_att, int64_t n_axis) {
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < n_att; c += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t a = c / n_axis, k = c - a * n_axis;
+    double z = 0.0;
+#pragma unroll
+    for (int jj = 0; jj < 4; ++jj) {
+      const int64_t w = k - jj;
+      if (w >= 0 && w <= n_axis - 4) {
+        double* p = z4 + 4 * (a * n_axis + w) + jj;
+        z += *p;
+        *p = 0.0;
+      }
+    }
+    zsh[c] += z;
+  }
+}
+static cudaError_t att_fold(const SysView& S, double* zsh, cudaStream_t s) {
+  if (!S.z4) return cudaSuccess;
+  k_att_fold<<<vec_grid(S.n_att, 148 * 4), kRedThreads, 0, s>>>(S.z4, zsh, S.n_att, S.n_axis);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh,
                          double* part, double* cpart, const DevState* st, cudaStream_t s) {
+  cudaError_t e;
 #ifdef LSQR_DIAG_EXPERIMENTS
   switch (diag_mode()) {
-    case 1: return fz3<R3_FUSED, 1>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 2: return fz3<R3_FUSED, 2>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 4: return fz3<R3_FUSED, 4>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 8: return fz3<R3_FUSED, 8>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 15: return fz3<R3_FUSED, 15>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 16: return fz3<R3_FUSED, 16>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    case 31: return fz3<R3_FUSED, 31>(S, grid, x, u, zA, zsh, part, cpart, st, s);
-    default: break;
+    case 1: e = fz3<R3_FUSED, 1>(S, grid, x, u, zA, zsh, part, cpart, st, s); break;
+    case 2: e = fz3<R3_FUSED, 2>(S, grid, x, u, zA, zsh, part, cpart, st, s); break;
+    case 4: e = fz3<R3_FUSED, 4>(S, grid, x, u, zA, zsh, part, cpart, st, s); break;
+    case 8: e = fz3<R3_FUSED, 8>(S, grid, x, u, zA, zsh, part, cpart, st, s); break;
+    case 15: e = fz3<R3_FUSED, 15>(S, grid, x, u, zA, zsh, part, cpart, st, s); break;
+    case 16: e = fz3<R3_FUSED, 16>(S, grid, x, u, zA, zsh, part, cpart, st, s); break;
+    case 31: e = fz3<R3_FUSED, 31>(S, grid, x, u, zA, zsh, part, cpart, st, s); break;
+    default: e = fz3<R3_FUSED, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s); break;
   }
+#else
+  e = fz3<R3_FUSED, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
 #endif
-  return fz3<R3_FUSED, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
+  return e != cudaSuccess ? e : att_fold(S, zsh, s);
 }
 
 cudaError_t launch_ap2_lean(const SysView& S, int grid, const double* u, double* zA, double* zsh, const DevState* st,
                             cudaStream_t s) {
-  return fz3<R3_AP2, 0>(S, grid, nullptr, const_cast<double*>(u), zA, zsh, nullptr, nullptr, st, s);
+  const cudaError_t e = fz3<R3_AP2, 0>(S, grid, nullptr, const_cast<double*>(u), zA, zsh, nullptr, nullptr, st, s);
+  return e != cudaSuccess ? e : att_fold(S, zsh, s);
 }
 
 cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const double* uc, double* zsh, double* part,
