@@ -99,6 +99,7 @@ struct lsqr_ctx {
   double* xatt4 = nullptr;      // the attitude gather copy of v (S.xatt4), kept by k_colupdate
   double* xatt4_api = nullptr;  // lsqr_aprod1's gather copy of its x (allocated on first use; pad entries unused)
   double* z4 = nullptr;         // attitude window accumulator of the fused kernel (S.z4), or nullptr
+  int32_t att_kmul = 4;         // gather-copy format (S.att_kmul): 4 knot, 16 window
   double* ingest = nullptr;  // lsqr_set_system staging (lazily allocated)
   double* uc_tmp = nullptr;  // k_post -> k_scalar constraint u_hat hand-over  // fused mode: astro z (A^T u_hat) and alpha^2 partials of k_vastro
   double *part_wa = nullptr, *part_ws = nullptr, *part_g1 = nullptr, *ar1 = nullptr, *uc = nullptr,
@@ -654,9 +655,10 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   AL(h->var, h->n_loc_cols);
   AL(h->D, h->n_loc_cols);
   AL(h->zsh, h->n_sh + 8);
-  AL(h->xatt4, 4 * n_axis);
   const bool use_z4 = n_att > 4096 && n_att <= kZ4MaxAtt && !getenv("LSQR_NO_Z4");  // 4096: kSmAttMax (smem copies)
   if (use_z4) AL(h->z4, 4 * n_att);
+  h->att_kmul = (n_att <= kZ4MaxAtt && !getenv("LSQR_KNOT_GATHER")) ? 16 : 4;  // window / knot gather format
+  AL(h->xatt4, (int64_t)h->att_kmul * n_axis);
   AL(h->part_rows, h->W);
   AL(h->part_a2, h->W);
   AL(h->cpart, std::max<int64_t>((int64_t)ch_row.size(), 1));
@@ -735,6 +737,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   S.n_csh = (int64_t)csh_idx.size(); S.csh_idx = d_cshi; S.csh_k = d_cshk; S.csh_e = d_cshe;
   S.scs_lo = scs_lo; S.scs_hi = scs_hi; S.scs_ptr = d_scsp; S.scs_k = d_scsk; S.scs_e = d_scse;
   S.xatt4 = h->xatt4;
+  S.att_kmul = h->att_kmul;
   S.z4 = h->z4;
   {  // bank-grouped instrumental slots only when every row kernel keeps the instrumental slice in shared memory
     InstrPerm probe;
@@ -745,7 +748,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   // zero-initialised state
   if (launch_fill(h->zsh, h->n_sh + 8, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (launch_fill(h->D, h->n_loc_cols, 1.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
-  if (launch_fill(h->xatt4, 4 * n_axis, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
+  if (launch_fill(h->xatt4, (int64_t)h->att_kmul * n_axis, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (h->z4 && launch_fill(h->z4, 4 * n_att, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   for (double* p : {h->v, h->w, h->x, h->var})
     if (launch_fill(p, h->n_loc_cols, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
@@ -957,7 +960,7 @@ int lsqr_aprod1(lsqr_t h, const double* x_dev, double* y_dev) {
   SysView& S = h->S;
   enter(h);
   // the attitude slice of x in the padded knot-major layout (32 B per knot, <= 32 MB), then one 256-bit load per lane
-  if (!h->xatt4_api) CKR(dalloc(h, &h->xatt4_api, 4 * h->n_axis));
+  if (!h->xatt4_api) CKR(dalloc(h, &h->xatt4_api, (int64_t)h->att_kmul * h->n_axis));
   CKL(h, launch_att_pack(S, x_dev, h->s, h->xatt4_api), "att_pack");
   CKL(h, launch_aprod1(AP1_PLAIN, S, h->grid, x_dev, y_dev, h->part_rows, h->cpart, h->st, h->s, h->xatt4_api),
       "aprod1");

@@ -117,6 +117,11 @@ struct SysView {
   // The fused kernel's attitude gather copy: xatt4[4k + a] = v[A0 + a n_axis + k] for a < 3, [4k + 3] = 0,
   // written by k_colupdate -- a lane's three axis values of knot k0 + j are one 32-B load (LDG.E.ENL2.256).
   double* xatt4;
+  // Window format of the same copy when the attitude slice is small enough (n_att <= kZ4MaxAtt; C2, C3):
+  // xatt4[16 k0 + 4 j + a] = v[A0 + a n_axis + k0 + j] -- every row's 4 lanes read ONE aligned 128-B line (4x the
+  // writes of the knot format, 128 B per knot).  att_kmul = 16 (window) or 4 (knot): a lane's address is
+  // xatt4 + att_kmul * k0 + 4 j.
+  int32_t att_kmul;
   // Attitude window accumulator of the fused kernel, or nullptr: z4[a][k0][j] (4 doubles per window
   // start k0, 32-B aligned) collects the 4 lanes' REDs of a row in one aligned sector; k_att_fold adds it into z_sh
   // after each pass.  Used when 4 n_att doubles stay well inside L2 (n_att <= kZ4MaxAtt) and the attitude slice is

@@ -425,7 +425,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int k0 = valid[q] ? rec.k0 : 0;
       xv[q][0] = ac.cj;
       if (G4) {
-        ldg_att4(xg4 + 4 * ((int64_t)k0 + j), xv[q][1], xv[q][2], xv[q][3]);
+        ldg_att4(xg4 + S.att_kmul * (int64_t)k0 + 4 * j, xv[q][1], xv[q][2], xv[q][3]);
       } else {
         xv[q][1] = __ldg(xatt0 + k0);
         xv[q][2] = __ldg(xatt1 + k0);
@@ -794,6 +794,7 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
   const int voff = r * kSlots * 8 + 48 * j, ioff = kFRows * kSlots * 8 + r * 16;
 #if LSQR_GATHER4
   const double* const xg4 = S.xatt4 + 4 * j;  // lane j gathers knot k0 + j (its three axis values, one load)
+  const int gmul = S.att_kmul;                  // 4: knot format, 16: window format (one 128-B line per row)
 #else
   const double* xatt0 = x + S.A0 + j;
   const double* xatt1 = xatt0 + S.n_axis;
@@ -881,7 +882,7 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
         P.g1 = P.g2 = P.g3 = 0.5;
       } else {
 #if LSQR_GATHER4
-        ldg_att4(xg4 + 4 * (int64_t)P.k0, P.g1, P.g2, P.g3);
+        ldg_att4(xg4 + gmul * (int64_t)P.k0, P.g1, P.g2, P.g3);
 #else
         P.g1 = __ldg(xatt0 + P.k0);
         P.g2 = __ldg(xatt1 + P.k0);
@@ -1488,9 +1489,24 @@ __global__ void __launch_bounds__(kRedThreads)
 
 // O-3e: v <- v/alpha (if pending); d = t3 w; var += d^2; x += t1 w; w = v + t2 w;  partials of ||w_new||^2 split
 // into the local astro columns (i < A0) and the replicated shared slice (i >= A0).
+// attitude column c (axis a, knot k) of v into the gather copy: knot format xg[4k + a]; window format
+// xg[16 w + 4 (k - w) + a] for every window start w in [k - 3, k] ∩ [0, n_axis - 4]
+__device__ __forceinline__ void att_put(double* __restrict__ xg, int kmul, int64_t n_axis, int64_t c, double v) {
+  const int64_t a = c / n_axis, k = c - a * n_axis;
+  if (kmul == 4) {
+    xg[4 * k + a] = v;
+    return;
+  }
+#pragma unroll
+  for (int jj = 0; jj < 4; ++jj) {
+    const int64_t w = k - jj;
+    if (w >= 0 && w <= n_axis - 4) xg[16 * w + 4 * jj + a] = v;
+  }
+}
+
 __global__ void __launch_bounds__(kRedThreads)
     k_colupdate(double* __restrict__ v, double* __restrict__ w, double* __restrict__ x, double* __restrict__ var,
-                int64_t n, int64_t A0, int64_t n_att, int64_t n_axis, double* __restrict__ xatt4,
+                int64_t n, int64_t A0, int64_t n_att, int64_t n_axis, double* __restrict__ xatt4, int kmul,
                 double* __restrict__ part_wa, double* __restrict__ part_ws, const DevState* __restrict__ st) {
   if (!st->col_enable) return;
   const double ia = st->v_pending ? st->inv_alpha : 1.0;
@@ -1509,10 +1525,7 @@ __global__ void __launch_bounds__(kRedThreads)
     } else {
       ws = fma(wnew, wnew, ws);
       const int64_t c = i - A0;
-      if (c < n_att) {  // the fused kernel's attitude gather copy: knot-major, padded to 4
-        const int64_t a = c / n_axis;
-        xatt4[4 * (c - a * n_axis) + a] = vi;
-      }
+      if (c < n_att) att_put(xatt4, kmul, n_axis, c, vi);  // the attitude gather copy
     }
   }
   wa = block_sum<kRedThreads>(wa);
@@ -1853,19 +1866,19 @@ cudaError_t launch_scalar(DevState* st, const double* part_astro, int64_t n_pa, 
 }
 cudaError_t launch_colupdate(const SysView& S, double* v, double* w, double* x, double* var, double* part_wa,
                              double* part_ws, int nblk, const DevState* st, cudaStream_t s) {
-  k_colupdate<<<nblk, kRedThreads, 0, s>>>(v, w, x, var, S.n_cols, S.A0, S.n_att, S.n_axis, S.xatt4, part_wa, part_ws,
-                                           st);
+  k_colupdate<<<nblk, kRedThreads, 0, s>>>(v, w, x, var, S.n_cols, S.A0, S.n_att, S.n_axis, S.xatt4, S.att_kmul,
+                                           part_wa, part_ws, st);
   return cudaGetLastError();
 }
 
-__global__ void k_att_pack(const double* __restrict__ v, int64_t n_att, int64_t n_axis, double* __restrict__ xatt4) {
-  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < n_att; c += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t a = c / n_axis;
-    xatt4[4 * (c - a * n_axis) + a] = v[c];
-  }
+__global__ void k_att_pack(const double* __restrict__ v, int64_t n_att, int64_t n_axis, double* __restrict__ xatt4,
+                           int kmul) {
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < n_att; c += (int64_t)gridDim.x * blockDim.x)
+    att_put(xatt4, kmul, n_axis, c, v[c]);
 }
 cudaError_t launch_att_pack(const SysView& S, const double* v, cudaStream_t s, double* dst) {
-  k_att_pack<<<vec_grid(S.n_att, 148 * 4), kRedThreads, 0, s>>>(v + S.A0, S.n_att, S.n_axis, dst ? dst : S.xatt4);
+  k_att_pack<<<vec_grid(S.n_att, 148 * 4), kRedThreads, 0, s>>>(v + S.A0, S.n_att, S.n_axis, dst ? dst : S.xatt4,
+                                                                 S.att_kmul);
   return cudaGetLastError();
 }
 cudaError_t launch_sum_to(const double* part, int64_t n, double* dst, cudaStream_t s) {
