@@ -100,6 +100,7 @@ struct lsqr_ctx {
   double* xatt4_api = nullptr;  // lsqr_aprod1's gather copy of its x (allocated on first use; pad entries unused)
   double* z4 = nullptr;         // attitude window accumulator of the fused kernel (S.z4), or nullptr
   int32_t att_kmul = 4;         // gather-copy format (S.att_kmul): 4 knot, 16 window
+  int32_t z4_kmul = 4;          // window-accumulator layout (S.z4_kmul)
   double* ingest = nullptr;  // lsqr_set_system staging (lazily allocated)
   double* uc_tmp = nullptr;  // k_post -> k_scalar constraint u_hat hand-over  // fused mode: astro z (A^T u_hat) and alpha^2 partials of k_vastro
   double *part_wa = nullptr, *part_ws = nullptr, *part_g1 = nullptr, *ar1 = nullptr, *uc = nullptr,
@@ -656,7 +657,11 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   AL(h->D, h->n_loc_cols);
   AL(h->zsh, h->n_sh + 8);
   const bool use_z4 = n_att > 4096 && n_att <= kZ4MaxAtt && !getenv("LSQR_NO_Z4");  // 4096: kSmAttMax (smem copies)
-  if (use_z4) AL(h->z4, 4 * n_att);
+  // z4[a][k0][j] (default); z4[k0][a][j] with LSQR_Z4_WINDOW_MAJOR (measured 3-7 % slower: the three RED instructions
+  // of a row then hit one line, serialising in the L2 atomic unit)
+  h->z4_kmul = getenv("LSQR_Z4_WINDOW_MAJOR") ? 16 : 4;
+  const int64_t z4_n = h->z4_kmul == 16 ? 16 * n_axis : 4 * n_att;
+  if (use_z4) AL(h->z4, z4_n);
   h->att_kmul = (n_att <= kZ4MaxAtt && !getenv("LSQR_KNOT_GATHER")) ? 16 : 4;  // window / knot gather format
   AL(h->xatt4, (int64_t)h->att_kmul * n_axis);
   AL(h->part_rows, h->W);
@@ -739,6 +744,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   S.xatt4 = h->xatt4;
   S.att_kmul = h->att_kmul;
   S.z4 = h->z4;
+  S.z4_kmul = h->z4_kmul;
   {  // bank-grouped instrumental slots only when every row kernel keeps the instrumental slice in shared memory
     InstrPerm probe;
     probe.init(n_instr, true);
@@ -749,7 +755,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   if (launch_fill(h->zsh, h->n_sh + 8, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (launch_fill(h->D, h->n_loc_cols, 1.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (launch_fill(h->xatt4, (int64_t)h->att_kmul * n_axis, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
-  if (h->z4 && launch_fill(h->z4, 4 * n_att, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
+  if (h->z4 && launch_fill(h->z4, z4_n, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   for (double* p : {h->v, h->w, h->x, h->var})
     if (launch_fill(p, h->n_loc_cols, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);
   if (launch_fill(h->u, h->n_loc_rows + 2, 0.0, h->s) != cudaSuccess) return bail(LSQR_ECUDA);

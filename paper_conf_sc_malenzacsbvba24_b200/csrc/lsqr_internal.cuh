@@ -127,6 +127,7 @@ struct SysView {
   // after each pass.  Used when 4 n_att doubles stay well inside L2 (n_att <= kZ4MaxAtt) and the attitude slice is
   // not privatised in shared memory.
   double* z4;
+  int32_t z4_kmul;  // 16: z4[k0][a (4)][j] (window-major, 128 B per window start); 4: z4[a][k0][j]
 };
 #ifndef LSQR_Z4_MAX_ATT
 #define LSQR_Z4_MAX_ATT (1 << 20)

@@ -801,12 +801,14 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
   const double* xatt2 = xatt1 + S.n_axis;
 #endif
   // attitude accumulator: axis-major z_att (lane j -> knot k0 + j of axis a), or, when S.z4 is set, the window
-  // accumulator z4[a][k0][j] (one 32-B-aligned sector per row and axis; folded into z_sh by k_att_fold)
+  // accumulator (folded into z_sh by k_att_fold): z4[k0][a][j] (z4_kmul = 16: a row's 12 REDs in one aligned 128-B
+  // line) or z4[a][k0][j] (z4_kmul = 4: one aligned 32-B sector per row and axis)
   const bool z4 = !SMATT && S.z4 != nullptr;
-  const int kmul = z4 ? 4 : 1;
+  const int kmul = z4 ? S.z4_kmul : 1;
+  const int64_t astride = !z4 ? S.n_axis : (kmul == 16 ? 4 : 4 * S.n_axis);
   double* zatt0 = (SMATT ? sh_za + (wid % arep) * S.n_att : (z4 ? S.z4 : zsh)) + j;
-  double* zatt1 = zatt0 + kmul * S.n_axis;
-  double* zatt2 = zatt1 + kmul * S.n_axis;
+  double* zatt1 = zatt0 + astride;
+  double* zatt2 = zatt1 + astride;
   double* const sh_zw = ZREP ? sh_z + (wid % zrep) * zstride : sh_z;  // this warp's z_instr copy
   const bool t5_ins = (j == 1 || j == 2);  // t=5 slot: lane 0 astro 4, lanes 1, 2 instr 4, 5, lane 3 global
   const int i5_shift = (j & 2) << 3;
@@ -1790,9 +1792,9 @@ static int diag_mode() {
 }
 #endif
 
-// z4 -> z_sh: z_att[a][k] += sum_j z4[a][k - j][j] (windows k - j in [0, n_axis - 4]); every z4 entry belongs to
+// z4 -> z_sh: z_att[a][k] += sum_j z4(w = k - j, a, j) (windows w in [0, n_axis - 4]); every z4 entry belongs to
 // exactly one column, which zeroes it after reading (the accumulator is clean for the next pass)
-__global__ void k_att_fold(double* __restrict__ z4, double* __restrict__ zsh, int64_t n_att, int64_t n_axis) {
+__global__ void k_att_fold(double* __restrict__ z4, double* __restrict__ zsh, int64_t n_att, int64_t n_axis, int kmul) {
   for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < n_att; c += (int64_t)gridDim.x * blockDim.x) {
     const int64_t a = c / n_axis, k = c - a * n_axis;
     double z = 0.0;
@@ -1800,7 +1802,7 @@ __global__ void k_att_fold(double* __restrict__ z4, double* __restrict__ zsh, in
     for (int jj = 0; jj < 4; ++jj) {
       const int64_t w = k - jj;
       if (w >= 0 && w <= n_axis - 4) {
-        double* p = z4 + 4 * (a * n_axis + w) + jj;
+        double* p = z4 + (kmul == 16 ? 16 * w + 4 * a : 4 * (a * n_axis + w)) + jj;
         z += *p;
         *p = 0.0;
       }
@@ -1810,7 +1812,7 @@ __global__ void k_att_fold(double* __restrict__ z4, double* __restrict__ zsh, in
 }
 static cudaError_t att_fold(const SysView& S, double* zsh, cudaStream_t s) {
   if (!S.z4) return cudaSuccess;
-  k_att_fold<<<vec_grid(S.n_att, 148 * 4), kRedThreads, 0, s>>>(S.z4, zsh, S.n_att, S.n_axis);
+  k_att_fold<<<vec_grid(S.n_att, 148 * 4), kRedThreads, 0, s>>>(S.z4, zsh, S.n_att, S.n_axis, S.z4_kmul);
   return cudaGetLastError();
 }
 
