@@ -940,7 +940,7 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
       un = valid ? uold : 0.0;  // aprod2: the u_hat aprod1 wrote
     }
     const double c1 = v[1] * un, c2 = v[2] * un, c3 = v[3] * un, c4v = v[4] * un, c5 = v[5] * un;
-    if (valid && !(DIAG & 2)) {  // per axis, the 4 lanes of a row hit 4 consecutive columns (one 32-B window)
+    if (valid && !(DIAG & 2)) {  // per axis, the 4 lanes of a row hit one 32-B window (z4: one aligned sector)
       const int ko = kmul * P.k0;
       atomicAdd(zatt0 + ko, c1);
       atomicAdd(zatt1 + ko, c2);
@@ -1489,8 +1489,6 @@ __global__ void __launch_bounds__(kRedThreads)
   if (host_flag) *reinterpret_cast<volatile int32_t*>(host_flag) = L.halted | (L.itn << 1);
 }
 
-// O-3e: v <- v/alpha (if pending); d = t3 w; var += d^2; x += t1 w; w = v + t2 w;  partials of ||w_new||^2 split
-// into the local astro columns (i < A0) and the replicated shared slice (i >= A0).
 // attitude column c (axis a, knot k) of v into the gather copy: knot format xg[4k + a]; window format
 // xg[16 w + 4 (k - w) + a] for every window start w in [k - 3, k] ∩ [0, n_axis - 4]
 __device__ __forceinline__ void att_put(double* __restrict__ xg, int kmul, int64_t n_axis, int64_t c, double v) {
@@ -1506,6 +1504,9 @@ __device__ __forceinline__ void att_put(double* __restrict__ xg, int kmul, int64
   }
 }
 
+// O-3e: v <- v/alpha (if pending); d = t3 w; var += d^2; x += t1 w; w = v + t2 w;  partials of ||w_new||^2 split
+// into the local astro columns (i < A0) and the replicated shared slice (i >= A0); the new v's attitude slice also
+// goes to the fused kernel's gather copy (att_put).
 __global__ void __launch_bounds__(kRedThreads)
     k_colupdate(double* __restrict__ v, double* __restrict__ w, double* __restrict__ x, double* __restrict__ var,
                 int64_t n, int64_t A0, int64_t n_att, int64_t n_axis, double* __restrict__ xatt4, int kmul,
