@@ -526,3 +526,33 @@ def test_lsqr_fused_edge_cases(avu, case):
         assert out["itn"] == 150
         assert rel(out["x"], ro["x"]) <= 1e-9, (case, fused, rel(out["x"], ro["x"]))
         assert abs(out["r1norm"] - ro["r1norm"]) <= 1e-9 * ro["r1norm"]
+
+
+@pytest.mark.parametrize("w", [W.C2, W.C1.replace(name="C1ia", n_att=4_200, n_instr=24_000, n_obs=120_000)],
+                         ids=["C2", "C1ia"])
+def test_attitude_layouts_agree(avu, w, monkeypatch):
+    """The attitude slice's device layouts -- window-format gather copy + window accumulator z4 (the default
+    for n_att <= 2^20), knot-format copy with axis-major REDs (C4/C5's), and window-major z4 -- give the same LSQR
+    (x after 150 fixed iterations within 1e-9, converged) and the same products (1e-13 of the terms' magnitudes)."""
+    import torch
+    runs = []
+    for env in ({}, {"LSQR_KNOT_GATHER": "1", "LSQR_NO_Z4": "1"}, {"LSQR_Z4_WINDOW_MAJOR": "1"}):
+        for k in ("LSQR_KNOT_GATHER", "LSQR_NO_Z4", "LSQR_Z4_WINDOW_MAJOR"):
+            monkeypatch.delenv(k, raising=False)
+        for k, v in env.items():
+            monkeypatch.setenv(k, v)
+        s = gpu_solver(avu, w)
+        s.precondition()
+        x = torch.linspace(-1, 1, s.n_local_cols, dtype=torch.float64, device="cuda")
+        y = torch.zeros(s.n_local_rows + s.n_constr, dtype=torch.float64, device="cuda")
+        s.aprod1(x, y)
+        x2 = torch.zeros_like(x)
+        s.aprod2(torch.linspace(-1, 1, y.numel(), dtype=torch.float64, device="cuda"), x2)
+        out = s.solve(itn_limit=150, atol=0, btol=0, conlim=0, fixed_count=True)
+        s.close()
+        runs.append((y.cpu().numpy(), x2.cpu().numpy(), out))
+    y0, x0, o0 = runs[0]
+    for y1, x1, o1 in runs[1:]:
+        assert np.allclose(y1, y0, rtol=1e-13, atol=1e-13 * np.abs(y0).max())
+        assert np.allclose(x1, x0, rtol=1e-13, atol=1e-13 * np.abs(x0).max())
+        assert rel(o1["x"], o0["x"]) <= 1e-9 and abs(o1["r1norm"] - o0["r1norm"]) <= 1e-10 * o0["r1norm"]
