@@ -310,18 +310,18 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
   }
   if (ev) cudaEventRecord(ev[0], s);
   if (fused) {
-    CKL(h, launch_fused(S, h->grid, h->v, h->u, h->zA, h->zsh, h->part_rows, h->cpart, h->st, s), "fused");
+    CKL(h, launch_fused(S, h->grid, h->v, h->u, h->zA, h->zsh, h->part_rows, h->cpart, h->st, s, multi), "fused");
   } else {
     CKL(h, launch_aprod1(AP1_LSQR, S, h->grid, h->v, h->u, h->part_rows, h->cpart, h->st, s, h->xatt4), "aprod1");
   }
   if (ev) cudaEventRecord(ev[1], s);
   if (!fused) {
     if (ev) cudaEventRecord(ev[2], s);
-    CKL(h, launch_ap2_lean(S, h->grid, h->u, h->zA, h->zsh, h->st, s), "aprod2");
+    CKL(h, launch_ap2_lean(S, h->grid, h->u, h->zA, h->zsh, h->st, s, multi), "aprod2");
     if (ev) cudaEventRecord(ev[3], s);
   }
   const int64_t n_b2 = fused ? h->grid : h->W;  // k_fused3 publishes one beta^2 partial per CTA, k_aprod1 per warp
-  if (!multi) {  // fused: 4 launches (rows, post = beta + v' everywhere, scalar, column update); two-pass: 5
+  if (!multi) {  // fused: 4 launches (rows, post = z4 fold + beta + v' everywhere, scalar, column update); two-pass: 5
     if (ev && fused) cudaEventRecord(ev[2], s);
     CKL(h, launch_post(S, h->v, h->zA, h->zsh, h->part_rows, n_b2, h->cpart, h->uc, h->uc_tmp, h->part_va, kG3,
                        h->st, s), "post");
@@ -354,7 +354,7 @@ int enqueue_iteration(lsqr_t h, cudaEvent_t* ev) {
 
 int kernels_per_iteration(lsqr_t h) {
   if (h->repro) return h->multi ? 15 : 7;
-  const int fold = h->z4 ? 1 : 0;  // k_att_fold after the row pass
+  const int fold = h->z4 && h->multi ? 1 : 0;  // k_att_fold after the row pass (P = 1: folded by k_post)
   if (!h->params.two_pass) return (h->multi ? 9 : 4) + fold;
   return (h->multi ? 10 : 5) + fold;
 }

@@ -175,14 +175,15 @@ cudaError_t launch_vshared(const SysView& S, double* vsh, double* zsh, double* p
                            int fused, cudaStream_t s);
 // NEXT-1 fused single pass (u_hat update + A^T u_hat in one read of A) and its astro column pass
 cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh,
-                         double* part, double* cpart, const DevState* st, cudaStream_t s);
+                         double* part, double* cpart, const DevState* st, cudaStream_t s, bool fold = true);
+// fold = false (single rank): k_post folds the window accumulator S.z4 into the attitude columns itself
 // lsqr_aprod2 after k_fused3<R3_AP2>: x_astro += zA + astro constraint entries . y_c; shared constraint entries -> z_sh
 cudaError_t launch_astro_add(const SysView& S, double* x, const double* zA, const double* yc, double* zsh,
                              int do_shared_constr, cudaStream_t s);
 // the two-pass iteration's aprod2 on the fused kernel's loop (k_fused3<R3_AP2>): z = A^T u_hat (unnormalised) into
 // zA / z_sh, the state the fused pass leaves (every instrumental-slice size: the IG regime covers large ones)
 cudaError_t launch_ap2_lean(const SysView& S, int grid, const double* u, double* zA, double* zsh, const DevState* st,
-                            cudaStream_t s);
+                            cudaStream_t s, bool fold = true);
 cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const double* uc, double* zsh, double* part,
                           int nblk, const DevState* st, int do_shared_constr, cudaStream_t s);
 // mode 0: x += z, 1: x = z; z zeroed
@@ -192,7 +193,8 @@ cudaError_t launch_scalar(DevState* st, const double* part_astro, int64_t n_pa, 
                           const double* ar2_alpha2, const double* ar1_wa, int init, int32_t* host_flag,
                           cudaStream_t s, const double* post_uc = nullptr, double* uc = nullptr,
                           double* ucn = nullptr, int nc = 0);
-// single-rank fused mode: beta (recomputed per block) + astro/shared v' + constraint terms in one kernel
+// single-rank fused mode: beta (recomputed per block) + astro/shared v' + constraint terms in one kernel; also folds
+// the row pass's attitude window accumulator S.z4 (the row pass was launched with fold = false)
 cudaError_t launch_post(const SysView& S, double* v, const double* zA, double* zsh, const double* part_rows,
                         int64_t n_part, const double* cpart, const double* uc, double* uc_tmp, double* part_a2,
                         int nblk, DevState* st, cudaStream_t s);

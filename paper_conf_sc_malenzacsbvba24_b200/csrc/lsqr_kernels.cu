@@ -1096,6 +1096,23 @@ __global__ void __launch_bounds__(kRedThreads)
 }
 
 
+// z4 -> z_sh: z_att[a][k] += sum_j z4(w = k - j, a, j) (windows w in [0, n_axis - 4]); every z4 entry belongs to
+// exactly one column, which zeroes it after reading (the accumulator is clean for the next pass)
+__device__ __forceinline__ double att_fold_col(double* __restrict__ z4, int64_t c, int64_t n_axis, int kmul) {
+  const int64_t a = c / n_axis, k = c - a * n_axis;
+  double z = 0.0;
+#pragma unroll
+  for (int jj = 0; jj < 4; ++jj) {
+    const int64_t w = k - jj;
+    if (w >= 0 && w <= n_axis - 4) {
+      double* p = z4 + (kmul == 16 ? 16 * w + 4 * a : 4 * (a * n_axis + w)) + jj;
+      z += *p;
+      *p = 0.0;
+    }
+  }
+  return z;
+}
+
 // Single-rank fused mode, after k_fused: beta (every block recomputes it from the deterministic partials; block 0
 // hands it to k_scalar through st->pb_*), then v' = z/beta - beta v on all local columns (astro from zA, shared
 // from z_sh, which is zeroed for the next iteration), constraint terms added per column, alpha^2 partials.
@@ -1166,6 +1183,7 @@ __global__ void __launch_bounds__(kRedThreads)
   double* vsh = v + S.A0;
   for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < S.n_sh; c += stride) {
     double z = zsh[c];
+    if (S.z4 && c < S.n_att) z += att_fold_col(S.z4, c, S.n_axis, S.z4_kmul);  // the row pass's window accumulator
     if (c >= S.scs_lo && c < S.scs_hi) {
       const int64_t q = c - S.scs_lo;
       for (int64_t e = S.scs_ptr[q]; e < S.scs_ptr[q + 1]; ++e) z += S.cval[S.scs_e[e]] * un_sh[S.scs_k[e]];
@@ -1793,23 +1811,9 @@ static int diag_mode() {
 }
 #endif
 
-// z4 -> z_sh: z_att[a][k] += sum_j z4(w = k - j, a, j) (windows w in [0, n_axis - 4]); every z4 entry belongs to
-// exactly one column, which zeroes it after reading (the accumulator is clean for the next pass)
 __global__ void k_att_fold(double* __restrict__ z4, double* __restrict__ zsh, int64_t n_att, int64_t n_axis, int kmul) {
-  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < n_att; c += (int64_t)gridDim.x * blockDim.x) {
-    const int64_t a = c / n_axis, k = c - a * n_axis;
-    double z = 0.0;
-#pragma unroll
-    for (int jj = 0; jj < 4; ++jj) {
-      const int64_t w = k - jj;
-      if (w >= 0 && w <= n_axis - 4) {
-        double* p = z4 + (kmul == 16 ? 16 * w + 4 * a : 4 * (a * n_axis + w)) + jj;
-        z += *p;
-        *p = 0.0;
-      }
-    }
-    zsh[c] += z;
-  }
+  for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < n_att; c += (int64_t)gridDim.x * blockDim.x)
+    zsh[c] += att_fold_col(z4, c, n_axis, kmul);
 }
 static cudaError_t att_fold(const SysView& S, double* zsh, cudaStream_t s) {
   if (!S.z4) return cudaSuccess;
@@ -1818,7 +1822,7 @@ static cudaError_t att_fold(const SysView& S, double* zsh, cudaStream_t s) {
 }
 
 cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u, double* zA, double* zsh,
-                         double* part, double* cpart, const DevState* st, cudaStream_t s) {
+                         double* part, double* cpart, const DevState* st, cudaStream_t s, bool fold) {
   cudaError_t e;
 #ifdef LSQR_DIAG_EXPERIMENTS
   switch (diag_mode()) {
@@ -1834,13 +1838,13 @@ cudaError_t launch_fused(const SysView& S, int grid, const double* x, double* u,
 #else
   e = fz3<R3_FUSED, 0>(S, grid, x, u, zA, zsh, part, cpart, st, s);
 #endif
-  return e != cudaSuccess ? e : att_fold(S, zsh, s);
+  return e != cudaSuccess || !fold ? e : att_fold(S, zsh, s);
 }
 
 cudaError_t launch_ap2_lean(const SysView& S, int grid, const double* u, double* zA, double* zsh, const DevState* st,
-                            cudaStream_t s) {
+                            cudaStream_t s, bool fold) {
   const cudaError_t e = fz3<R3_AP2, 0>(S, grid, nullptr, const_cast<double*>(u), zA, zsh, nullptr, nullptr, st, s);
-  return e != cudaSuccess ? e : att_fold(S, zsh, s);
+  return e != cudaSuccess || !fold ? e : att_fold(S, zsh, s);
 }
 
 cudaError_t launch_vastro(const SysView& S, double* v, const double* zA, const double* uc, double* zsh, double* part,
