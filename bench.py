@@ -499,6 +499,8 @@ def run_ours(args):
         "gpu_launches": int(max_over_ranks(r["launches"])),
         "timing": {"value_pass": "lsqr_iterate x K (CUDA graph replay, the lsqr_solve path), events around the K "
                                  "iterations", "roofline_pass": "lsqr_iterate_timed x K (events around every kernel)",
+                   "note": "the two passes run back to back in the clock-sampled region; under the power cap their "
+                           "SM clocks can differ by ~1 %, so avg_launch_ms can exceed ms_per_step",
                    "instrumented_ms_per_step": round(t_instr_ms / K, 5)},
         "clocks": clk.summary(),
         "e2e": e2e,
