@@ -140,6 +140,9 @@ enum {
 
 /* ---------------------------------------------------------------- meta / host-only helpers (no GPU needed) */
 int lsqr_abi_version(void);
+/* Hash of the library's sources (csrc/*.cu, *.cuh and this header) it was built from, as 16 lower-case hex digits;
+ * static storage, never NULL.  The Python binding compares it with the sources on disk and refuses a stale build. */
+const char* lsqr_build_id(void);
 const char* lsqr_strerror(int status);
 
 /* Observations per star of the synthetic generator (O-GEN): uniform q = floor(n_obs/n_stars) (+1 for the first

@@ -56,6 +56,7 @@ class Result(C.Structure):
 
 EXPORTS = {
     "lsqr_abi_version": (C.c_int, []),
+    "lsqr_build_id": (C.c_char_p, []),
     "lsqr_strerror": (C.c_char_p, [C.c_int]),
     "lsqr_last_error": (C.c_char_p, [vp]),
     "lsqr_synth_obs_per_star": (C.c_int, [u64, i64, i64, i32, vp]),
@@ -90,7 +91,8 @@ def lib_path() -> str:
 
 
 def lib(build_if_missing: bool = True):
-    """Loads liblsqr_avugsr.so (building it first when the sources are newer and nvcc is available)."""
+    """Loads liblsqr_avugsr.so, building it first when it is missing or was built from other sources (its embedded
+    build id differs from the hash of csrc/ and the header); refuses a library whose id does not match."""
     global _lib
     with _lock:
         if _lib is None:
@@ -104,6 +106,10 @@ def lib(build_if_missing: bool = True):
                 f = getattr(L, name)
                 f.restype = res
                 f.argtypes = args
+            bid, want = L.lsqr_build_id().decode(), _build.source_hash()
+            if bid != want:  # a stale library must never stand in for the sources under test
+                raise RuntimeError(f"{_build.LIB} was built from other sources (build id {bid}, sources {want}); "
+                                   "rebuild it (__graft_entry__.build())")
             _lib = L
     return _lib
 

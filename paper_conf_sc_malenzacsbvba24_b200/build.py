@@ -1,6 +1,7 @@
 """Builds liblsqr_avugsr.so in-tree with nvcc for sm_100a (no JIT cache: the .so travels with the repo snapshot)."""
 from __future__ import annotations
 
+import hashlib
 import os
 import subprocess
 import sys
@@ -36,13 +37,35 @@ def _nvcc() -> str:
     return "nvcc"
 
 
-def needs_build() -> bool:
-    if not os.path.exists(LIB):
-        return True
-    t = os.path.getmtime(LIB)
-    deps = [os.path.join(CSRC, s) for s in SOURCES] + [h if os.path.isabs(h) else os.path.join(CSRC, h)
+def _deps() -> list[str]:
+    return [os.path.join(CSRC, s) for s in SOURCES] + [h if os.path.isabs(h) else os.path.join(CSRC, h)
                                                       for h in HEADERS]
-    return any(os.path.getmtime(d) > t for d in deps)
+
+
+def source_hash() -> str:
+    """16 hex digits of SHA-256 over the library's sources and headers (embedded in the .so as lsqr_build_id)."""
+    h = hashlib.sha256()
+    for d in _deps():
+        h.update(os.path.basename(d).encode() + b"\0")
+        with open(d, "rb") as f:
+            h.update(f.read())
+    return h.hexdigest()[:16]
+
+
+def built_id(path: str = LIB) -> str | None:
+    """The build id embedded in the .so (its LSQR_BUILD_ID marker), read from the file without loading it."""
+    try:
+        with open(path, "rb") as f:
+            data = f.read()
+    except OSError:
+        return None
+    i = data.find(b"LSQR_BUILD_ID=")
+    return data[i + 14:i + 30].decode("ascii", "replace") if i >= 0 else None
+
+
+def needs_build() -> bool:
+    """True when the library is missing or was built from other sources than those on disk."""
+    return built_id() != source_hash()
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
@@ -50,7 +73,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"
     cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC,-O2",
-           "-Xptxas", "-warn-spills", "-I", os.path.join(ROOT, "include"), "-I", CSRC, "-I", _nccl_include(),
+           "-Xptxas", "-warn-spills", f"-DLSQR_SOURCE_HASH=\"{source_hash()}\"",
+           "-I", os.path.join(ROOT, "include"), "-I", CSRC, "-I", _nccl_include(),
            "-o", tmp] + [os.path.join(CSRC, s) for s in SOURCES] + ["-ldl"]
     extra = os.environ.get("LSQR_NVCC_EXTRA", "").split()  # experiment builds only (e.g. -DLSQR_DIAG_EXPERIMENTS)
     cmd[1:1] = extra

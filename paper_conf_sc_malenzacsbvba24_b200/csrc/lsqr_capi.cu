@@ -389,6 +389,13 @@ extern "C" {
 
 int lsqr_abi_version(void) { return LSQR_ABI_VERSION; }
 
+#ifndef LSQR_SOURCE_HASH
+#define LSQR_SOURCE_HASH "0000000000000000"
+#endif
+// the marker lets build.py read the id from the .so file without loading it
+static const char kBuildId[] = "LSQR_BUILD_ID=" LSQR_SOURCE_HASH;
+const char* lsqr_build_id(void) { return kBuildId + 14; }
+
 const char* lsqr_strerror(int status) {
   switch (status) {
     case LSQR_OK: return "ok";

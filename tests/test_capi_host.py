@@ -98,6 +98,20 @@ def test_missing_extension_fails_loudly(monkeypatch, tmp_path):
         _capi.lib(build_if_missing=False)
 
 
+def test_stale_library_is_refused(monkeypatch):
+    """The library embeds the hash of the sources it was built from (lsqr_build_id); a library built from other
+    sources is rebuilt (needs_build) or, when building is not allowed, refused -- never loaded silently."""
+    from paper_conf_sc_malenzacsbvba24_b200 import _capi, build as _build
+    L = _capi.lib()
+    assert L.lsqr_build_id().decode() == _build.source_hash() == _build.built_id()
+    assert not _build.needs_build()
+    monkeypatch.setattr(_build, "source_hash", lambda: "f" * 16)  # as if a source had changed since the build
+    assert _build.needs_build()
+    monkeypatch.setattr(_capi, "_lib", None)
+    with pytest.raises(RuntimeError, match="other sources"):
+        _capi.lib(build_if_missing=False)
+
+
 def test_product_package_never_touches_the_oracle():
     """The product path (package sources, CUDA, C ABI header) shares no code with oracle/ and does not import it."""
     import glob
