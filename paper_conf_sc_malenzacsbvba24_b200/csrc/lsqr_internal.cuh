@@ -123,8 +123,8 @@ struct SysView {
   // xatt4 + att_kmul * k0 + 4 j.
   int32_t att_kmul;
   // Attitude window accumulator of the fused kernel, or nullptr: z4[a][k0][j] (4 doubles per window
-  // start k0, 32-B aligned) collects the 4 lanes' REDs of a row in one aligned sector; k_att_fold adds it into z_sh
-  // after each pass.  Used when 4 n_att doubles stay well inside L2 (n_att <= kZ4MaxAtt) and the attitude slice is
+  // start k0, 32-B aligned) collects the 4 lanes' REDs of a row in one aligned sector; k_post (P = 1) or k_att_fold
+  // (P > 1, the lsqr_aprod2 API) folds it into the attitude columns after each pass and zeroes it.  Used when 4 n_att doubles stay well inside L2 (n_att <= kZ4MaxAtt) and the attitude slice is
   // not privatised in shared memory.
   double* z4;
   int32_t z4_kmul;  // 16: z4[k0][a (4)][j] (window-major, 128 B per window start); 4: z4[a][k0][j]

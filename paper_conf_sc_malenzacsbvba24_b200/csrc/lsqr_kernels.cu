@@ -801,7 +801,7 @@ __global__ void __launch_bounds__(kFWarps * 32, 1)
   const double* xatt2 = xatt1 + S.n_axis;
 #endif
   // attitude accumulator: axis-major z_att (lane j -> knot k0 + j of axis a), or, when S.z4 is set, the window
-  // accumulator (folded into z_sh by k_att_fold): z4[k0][a][j] (z4_kmul = 16: a row's 12 REDs in one aligned 128-B
+  // accumulator (folded by k_post, or into z_sh by k_att_fold): z4[k0][a][j] (z4_kmul = 16: a row's 12 REDs in one aligned 128-B
   // line) or z4[a][k0][j] (z4_kmul = 4: one aligned 32-B sector per row and axis)
   const bool z4 = !SMATT && S.z4 != nullptr;
   const int kmul = z4 ? S.z4_kmul : 1;
