@@ -167,9 +167,9 @@ def cpu_baseline(w, iters=3, repro=False, all_cores=True):
               f"full-system s/iteration extrapolated as "
               f"t_iter + (P-1) * t(aprod1 + aprod2) on the sample (setup {t_setup:.1f} s excluded)")
     out = {"value": serial["value"], "unit": UNIT, "cores": 1, "kind": "oracle",
-           "sample": sample, "serial": serial, "cpu_model": _cpu_model(), "host_cores": os.cpu_count()}
+           "sample": sample, "serial": serial, "cpu_model": _cpu_model(), "host_cores": _host_cores()}
     if all_cores and not repro:
-        r = oracle.time_lsqr_omp(S, iters)
+        r = oracle.time_lsqr_omp(S, iters, threads=_host_cores())
         L = oracle.omp_lib()
         fns = (lambda x, y: L.orc_omp_aprod1(ctypes.byref(S.S), oracle._p(x), oracle._p(y)),
                lambda y, x: L.orc_omp_aprod2(ctypes.byref(S.S), oracle._p(y), oracle._p(x)))
@@ -181,6 +181,15 @@ def cpu_baseline(w, iters=3, repro=False, all_cores=True):
         out.update(value=omp["value"], cores=omp["cores"], build="all-core OpenMP timing build (value, cores); "
                    "the serial checker as it stands under 'serial'", all_cores=omp)
     return out
+
+
+def _host_cores():
+    """Cores this process may run on (the OpenMP timing build uses all of them, whatever OMP_NUM_THREADS says:
+    torchrun exports OMP_NUM_THREADS=1 to every rank, and only rank 0 runs the oracle)."""
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
 
 
 def _mem_available():
@@ -273,14 +282,17 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
-    w = workload_of(args)
+    n = int(os.environ.get("WORLD_SIZE", str(args.gpus)))
+    base = workload_of(args)
+    # the whole job our arm times at this N (weak: n x the configuration; strong: the configuration)
+    w = (base.per_gpu(n) if (n > 1 and args.scaling == "weak") else base).replace(name=base.name)
     import ctypes
     import oracle
     t0 = time.perf_counter()
     S, P = oracle_sample(w)
     S.apply_precond()
     setup = time.perf_counter() - t0
-    r = oracle.time_lsqr_omp(S, args.warmup + args.steps)
+    r = oracle.time_lsqr_omp(S, args.warmup + args.steps, threads=_host_cores())
     per = r["per_iter_s"][args.warmup:]
     L = oracle.omp_lib()
     t_pr = _time_products(S, (lambda x, y: L.orc_omp_aprod1(ctypes.byref(S.S), oracle._p(x), oracle._p(y)),
@@ -291,14 +303,15 @@ def run_reference(args):
     sample = (f"rows of shard 0 of {P} of {w.name} ({S.n_rows} of {w.n_obs} rows; all {S.n_cols} columns), "
               f"{len(per)} LSQR iterations after {args.warmup} warm-up (mean {t_it:.4f} s on the sample); "
               f"full-system s/iteration = t_iter + (P-1) * t(aprod1 + aprod2) = {v:.3f} (setup {setup:.1f} s excluded)")
-    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": n,
             "steps": len(per), "warmup": args.warmup, "ms_per_step": v * 1e3, "higher_is_better": False,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": config_block(w, 1, args, {"note": "CPU oracle, all-core OpenMP timing build "
-                                                        "(oracle/omp_timing.c), on the host; rank 0 only"}),
+            "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": config_block(w, n, args, {"note": "CPU oracle, all-core OpenMP timing build "
+                                                        "(oracle/omp_timing.c), on the host; rank 0 only, timing "
+                                                        "the whole job of this N"}),
             "cpu_baseline": {"value": v, "unit": UNIT, "cores": r["threads"], "kind": "oracle",
                              "build": "all-core OpenMP timing build (oracle/omp_timing.c)", "sample": sample,
-                             "cpu_model": _cpu_model(), "host_cores": os.cpu_count()},
+                             "cpu_model": _cpu_model(), "host_cores": _host_cores()},
             "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     emit(line)
     return 0

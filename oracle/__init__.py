@@ -357,6 +357,7 @@ def omp_lib():
             L = C.CDLL(build_omp())
             vp, i64, i32, d = C.c_void_p, C.c_int64, C.c_int32, C.c_double
             L.orc_omp_threads.restype = C.c_int
+            L.orc_omp_set_threads.argtypes = [C.c_int]
             for f in (L.orc_omp_aprod1, L.orc_omp_aprod2):
                 f.argtypes = [C.POINTER(SysStruct), vp, vp]
             L.orc_lsqr.restype = C.c_int
@@ -366,11 +367,14 @@ def omp_lib():
     return _omp
 
 
-def time_lsqr_omp(sysm: System, iters: int) -> dict:
+def time_lsqr_omp(sysm: System, iters: int, threads: int | None = None) -> dict:
     """TIMING ONLY: `iters` fixed-count LSQR iterations of the all-core variant on an already preconditioned
-    System; returns per-iteration wall times (the first, which includes O-1, is dropped) and the thread count."""
+    System; returns per-iteration wall times (the first, which includes O-1, is dropped) and the thread count.
+    threads: OpenMP threads for this and later calls from this thread (None: the OpenMP default)."""
     import time
     L = omp_lib()
+    if threads:
+        L.orc_omp_set_threads(int(threads))
     stamps = []
 
     def _tr(stp, u, v, w_, xx, vv, _ctx):

@@ -19,6 +19,10 @@
 #include <omp.h>
 
 int orc_omp_threads(void) { return omp_get_max_threads(); }
+/* thread count of the parallel loops that follow (n > 0); torchrun exports OMP_NUM_THREADS=1 to every rank */
+void orc_omp_set_threads(int n) {
+  if (n > 0) omp_set_num_threads(n);
+}
 
 void orc_omp_aprod1(const orc_sys* S, const double* x, double* y) {
 #pragma omp parallel for schedule(static)

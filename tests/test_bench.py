@@ -29,6 +29,17 @@ def test_reference_arm_cpu():
     assert d["config"]["workload"] == "C1"
 
 
+def test_reference_arm_two_ranks_cpu():
+    """Under torchrun (N > 1) rank 0 alone times the oracle on the whole job our arm times at that N (weak: N x the
+    configuration) on all host cores (torchrun exports OMP_NUM_THREADS=1); the other ranks exit 0 without work."""
+    d = _run(["-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr", "127.0.0.1",
+              "--master-port", "29545", "bench.py", "--impl", "reference", "--gpus", "2", "--config", "C1",
+              "--steps", "3", "--warmup", "3"])
+    assert d["impl"] == "reference" and d["n_gpus"] == 2 and d["scaling"] == "weak"
+    assert d["config"]["total_rows"] == 40_000 and d["config"]["n_obs_per_gpu"] == 20_000
+    assert d["cpu_baseline"]["cores"] == d["cpu_baseline"]["host_cores"] >= 1
+
+
 @pytest.mark.gpu
 def test_bench_line_gpu(cuda_device):
     d = _run(["bench.py", "--config", "C1", "--steps", "5", "--warmup", "3", "--cpu-iters", "2"])
