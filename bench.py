@@ -330,6 +330,10 @@ def run_ours(args):
     torch.cuda.set_device(local)
     multi = world > 1
     use_nccl = args.comm == "nccl"
+    if multi and use_nccl:
+        # NCCL's own init log on stderr (communicator size, NVLS / ring / tree choice) so the launch can be audited;
+        # the JSON line goes to stdout
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
     if multi:
         if use_nccl:
             dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", local))
