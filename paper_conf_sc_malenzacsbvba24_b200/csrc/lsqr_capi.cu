@@ -755,7 +755,7 @@ int lsqr_create(int64_t n_stars, int64_t n_obs, int64_t n_att, int64_t n_instr, 
   {  // bank-grouped instrumental slots only when every row kernel keeps the instrumental slice in shared memory
     InstrPerm probe;
     probe.init(n_instr, true);
-    S.ip.init(n_instr, probe.slots() <= kInstrSmemMax);
+    S.ip.init(n_instr, probe.slots() <= kInstrSmemMax && !getenv("LSQR_NO_INSTR_PERM"));  // env: A/B only
   }
 
   // zero-initialised state
