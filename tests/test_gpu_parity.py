@@ -393,6 +393,42 @@ def test_lsqr_special_cases(avu):
     s.close()
 
 
+@pytest.mark.parametrize("w", [W.micro(n_stars=1, obs=9, jitter=0, seed=21),
+                               W.micro(n_stars=3, obs=1, jitter=0, seed=22),
+                               W.micro(n_stars=5, obs=3, n_ext=2, seed=23),
+                               W.micro(n_stars=9, obs=1, n_glob=0, seed=24)],
+                         ids=["1star", "1row_per_star", "constraints", "noglob"])
+def test_lsqr_tiny_systems(avu, w):
+    """Fewer rows than one 8-row group / one warp's stage, one star, one row per star (m < n: LSQR from x0 = 0
+    converges to the minimum-norm solution on both sides): products 1e-13 of the terms, converged x 1e-8, both
+    variants."""
+    import torch
+    S = oracle.System(w)
+    A = abs_system(S)
+    rng = np.random.default_rng(w.seed)
+    x = rng.standard_normal(S.n_cols)
+    yo = np.zeros(S.m_local); S.aprod1(x, yo)
+    ya = np.zeros(S.m_local); A.aprod1(np.abs(x), ya)
+    y = rng.standard_normal(S.m_local)
+    xo = np.zeros(S.n_cols); S.aprod2(y, xo)
+    xa = np.zeros(S.n_cols); A.aprod2(np.abs(y), xa)
+    ro = oracle.solve_system(oracle.System(w), itn_limit=300, atol=1e-13, btol=1e-13, conlim=0, fixed_count=False)
+    for fused in (True, False):
+        s = gpu_solver(avu, w)
+        yg = torch.zeros(S.m_local, dtype=torch.float64, device="cuda")
+        s.aprod1(torch.tensor(x, device="cuda"), yg)
+        assert np.all(np.abs(yg.cpu().numpy() - yo) <= 1e-13 * (ya + 1e-300))
+        xg = torch.zeros(S.n_cols, dtype=torch.float64, device="cuda")
+        s.aprod2(torch.tensor(y, device="cuda"), xg)
+        assert np.all(np.abs(xg.cpu().numpy() - xo) <= 1e-13 * (xa + 1e-300))
+        s.close()
+        s = gpu_solver(avu, w)
+        s.precondition()
+        out = s.solve(itn_limit=300, atol=1e-13, btol=1e-13, conlim=0, fixed_count=False, fused=fused)
+        s.close()
+        assert out["istop"] in (1, 2) and rel(out["x"], ro["x"]) <= 1e-8, (fused, out["istop"], rel(out["x"], ro["x"]))
+
+
 def test_lsqr_damped(avu):
     w = W.micro(n_stars=30, obs=25, seed=11)
     s = gpu_solver(avu, w)
