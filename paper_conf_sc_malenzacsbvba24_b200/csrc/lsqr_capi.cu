@@ -1027,6 +1027,8 @@ int lsqr_init(lsqr_t h, const lsqr_solve_params* p) {
   CKC(h, cudaMemcpyAsync(h->st, &st0, sizeof st0, cudaMemcpyHostToDevice, h->s));
   for (double* q : {h->v, h->w, h->x, h->var}) CKL(h, launch_fill(q, h->n_loc_cols, 0.0, h->s), "fill");
   CKL(h, launch_fill(h->zsh, h->n_sh + 8, 0.0, h->s), "fill");
+  if (h->z4)  // the window accumulator is clean after every pass; re-zeroed here in case a solve ended mid-pass
+    CKL(h, launch_fill(h->z4, h->z4_kmul == 16 ? 16 * h->S.n_axis : 4 * h->S.n_att, 0.0, h->s), "fill");
   if (h->repro) {  // NEXT-4 O-1
     CKC(h, cudaMemsetAsync(h->rzd, 0, sizeof(long long) * repro_digits_per_value() * h->n_loc_cols, h->s));
     CKC(h, cudaMemsetAsync(h->rsd, 0, sizeof(long long) * repro_sd_size(h->n_constr), h->s));

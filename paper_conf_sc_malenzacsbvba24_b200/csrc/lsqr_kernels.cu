@@ -1168,7 +1168,13 @@ __global__ void __launch_bounds__(kRedThreads)
   __syncthreads();
   if (blockIdx.x == 0 && threadIdx.x < nc) uc_tmp[threadIdx.x] = un_sh[threadIdx.x];
   const double beta = bsh[0], ib = bsh[1];
-  if (bsh[2] == 0.0) return;  // beta == 0: v is left unchanged (P&S step b skipped)
+  if (bsh[2] == 0.0) {  // beta == 0: v is left unchanged (P&S step b skipped); leave the accumulators clean
+    for (int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; c < S.n_sh; c += (int64_t)gridDim.x * blockDim.x) {
+      if (S.z4 && c < S.n_att) att_fold_col(S.z4, c, S.n_axis, S.z4_kmul);
+      zsh[c] = 0.0;
+    }
+    return;
+  }
   double a2 = 0.0;
   const int64_t na = 5 * S.n_stars;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
