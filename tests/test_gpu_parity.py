@@ -429,6 +429,46 @@ def test_lsqr_tiny_systems(avu, w):
         assert out["istop"] in (1, 2) and rel(out["x"], ro["x"]) <= 1e-8, (fused, out["istop"], rel(out["x"], ro["x"]))
 
 
+def test_handles_are_independent(avu):
+    """Two live handles in one process (different shared-slice regimes: C1c's shared-memory attitude copies and a
+    z4/window-copy system), stepped alternately, and two handles solved concurrently from two threads, give the
+    results each gives alone (no state shared between handles beyond the per-device kernel attributes)."""
+    import threading
+    wa = W.C1C
+    wb = W.C1.replace(name="C1z", n_att=6_000, n_instr=6_000)
+    kw = dict(itn_limit=600, atol=1e-12, btol=1e-12, conlim=0)  # converged: rounding-order independent to ~1e-9
+    ref = {}
+    for w in (wa, wb):
+        s = gpu_solver(avu, w)
+        s.precondition()
+        ref[w.name] = s.solve(**kw)
+        s.close()
+    sa, sb = gpu_solver(avu, wa), gpu_solver(avu, wb)
+    for s in (sa, sb):
+        s.precondition()
+        s.init(**kw)
+    for _ in range(12):  # iterations after istop are no-ops
+        sa.iterate(50)
+        sb.iterate(50)
+    outs = {wa.name: sa.finalize(), wb.name: sb.finalize()}
+    sa.close(); sb.close()
+    got = {}
+
+    def run(w):
+        import torch
+        torch.cuda.set_device(0)
+        s = gpu_solver(avu, w)
+        s.precondition()
+        got[w.name] = s.solve(**kw)
+        s.close()
+    th = [threading.Thread(target=run, args=(w,)) for w in (wa, wb)]
+    for t in th: t.start()
+    for t in th: t.join()
+    for name in (wa.name, wb.name):
+        for o in (outs[name], got[name]):
+            assert o["istop"] in (1, 2) and rel(o["x"], ref[name]["x"]) <= 1e-8, (name, rel(o["x"], ref[name]["x"]))
+
+
 def test_lsqr_damped(avu):
     w = W.micro(n_stars=30, obs=25, seed=11)
     s = gpu_solver(avu, w)
